@@ -1,0 +1,382 @@
+"""Benchmark: 1D C2C FFT GFLOP/s = 5 N log2 N / t of the FMM-FFT (BASELINE.json "metric").
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl fmmfft|reference] [--workload NAME]
+
+N = 1 runs configs[1] (cfg2: N = 2^20 complex64, P = 64, B = 2, Q = 16 on one GPU).
+N > 1 (launched by torch.distributed.run, one rank per GPU over NCCL) runs configs[2]
+(cfg3: N = 2^26 complex64, P = 16 G, B = 4, Q = 16) — strong scaling, one global FFT.
+
+A "step" is one fmmfft_execute of the whole hot path (Algorithm 1 + POST + the distributed 2D
+FFT) on inputs resident in HBM. Between steps L2 is flushed (a 256 MiB write, outside the
+timed events). Each step is timed with CUDA events on the plan's stream; the K-step total is
+bracketed by barrier + synchronize and the max over ranks is reported. Rank 0 prints ONE JSON
+line. --impl reference times the CPU float64 oracle (oracle/) on host cores instead.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+WORKLOADS = {
+    # name: (N, precision, P(G), B, Q, M_L, description)
+    "cfg1": (1 << 12, "c128", lambda G: 16, 2, 16, 64, "configs[0]: N=2^12 complex128, P=16, B=2, Q=16"),
+    "cfg2": (1 << 20, "c64", lambda G: 64, 2, 16, 64, "configs[1]: N=2^20 complex64, P=64, G=1, B=2, Q=16"),
+    "cfg3": (1 << 26, "c64", lambda G: 16 * G, 4, 16, 64, "configs[2]: N=2^26 complex64, P=16G, B=4, Q=16"),
+    "cfg4": (1 << 28, "c128", lambda G: 64 * G, 2, 24, 64, "configs[3]: N=2^28 complex128, P=64G, B=2, Q=24"),
+}
+
+NVML_REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+                0x20: "sync_boost", 0x40: "sw_thermal_slowdown", 0x80: "hw_thermal_slowdown",
+                0x100: "hw_power_brake_slowdown", 0x200: "display_clock_setting"}
+
+
+def flops_fft(N: int) -> float:
+    return 5.0 * N * math.log2(N)
+
+
+def near_up_flops(N, P, B, Q, M_L, G, C=2):
+    """Algorithmic flops of one near_up launch (S2T + S2M, §5.1), per rank."""
+    L = int(round(math.log2(N // (P * M_L))))
+    s2t = 6 * C * M_L * M_L * 2 ** L * (P - 1) / G
+    s2m = 2 * C * M_L * 2 ** L * (P - 1) * Q / G
+    return s2t + s2m
+
+
+class ClockSampler:
+    """NVML sampling of SM clock and throttle reasons while the timed loop runs."""
+
+    def __init__(self, device_index: int, period_s: float = 0.01):
+        self.samples = []
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self._h = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self._nv = pynvml
+            self._h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self._h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self._h = None
+        self.period = period_s
+        self.t = threading.Thread(target=self._run, daemon=True)
+        self.active = threading.Event()
+
+    def _run(self):
+        while not self._stop.is_set():
+            if self.active.is_set():
+                try:
+                    mhz = self._nv.nvmlDeviceGetClockInfo(self._h, self._nv.NVML_CLOCK_SM)
+                    rs = self._nv.nvmlDeviceGetCurrentClocksEventReasons(self._h)
+                    self.samples.append((mhz, rs))
+                except Exception:
+                    pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self._h is not None:
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._h is not None:
+            self.t.join(timeout=2)
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": [], "samples": 0}
+        mask = 0
+        for _, r in self.samples:
+            mask |= r
+        return {"sm_mhz": statistics.median(m for m, _ in self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": [n for b, n in NVML_REASONS.items() if mask & b and b != 0x1],
+                "samples": len(self.samples)}
+
+
+def load_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+def load_traffic(workload: str, G: int):
+    """Per-launch DRAM bytes of near_up from the committed ncu --set full summary, if any."""
+    try:
+        d = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
+        e = d.get(f"{workload}_G{G}")
+        return e and e.get("near_up_dram_bytes")
+    except Exception:
+        return None
+
+
+# ------------------------------------------------------------------------------ CPU oracle legs
+def oracle_sample(workload: str, G: int, budget_s: float):
+    """Time the CPU float64 oracle on a bounded sample of the workload: the full problem if one
+    run fits in the budget, else the same (P, B, Q, M_L) at the largest N' that does."""
+    import numpy as np
+    try:
+        from threadpoolctl import threadpool_limits
+        lim = threadpool_limits(1)
+    except Exception:
+        lim = None
+    import synth_inputs as SI
+    from oracle import fmmfft_oracle as O
+    N, prec, Pf, B, Q, M_L, _ = WORKLOADS[workload]
+    P = Pf(G)
+    # smallest legal N' for these parameters: L = B
+    n_min = P * M_L * (1 << B)
+    Ns = n_min
+    x = SI.complex_uniform(0, Ns)
+    t0 = time.perf_counter()
+    O.fmmfft(x, P, B, Q, M_L)
+    t = time.perf_counter() - t0
+    while Ns < N and t * 2.2 < budget_s:
+        Ns *= 2
+        x = SI.complex_uniform(0, Ns)
+        t0 = time.perf_counter()
+        O.fmmfft(x, P, B, Q, M_L)
+        t = time.perf_counter() - t0
+    del lim
+    return Ns, P, B, Q, M_L, x
+
+
+def time_oracle(Ns, P, B, Q, M_L, x, reps_budget_s):
+    from oracle import fmmfft_oracle as O
+    try:
+        from threadpoolctl import threadpool_limits
+        lim = threadpool_limits(1)
+    except Exception:
+        lim = None
+    times = []
+    t_start = time.perf_counter()
+    while True:
+        t0 = time.perf_counter()
+        O.fmmfft(x, P, B, Q, M_L)
+        times.append(time.perf_counter() - t0)
+        if time.perf_counter() - t_start > reps_budget_s:
+            break
+    del lim
+    return times
+
+
+def cpu_baseline(workload: str, G: int, budget_s: float = 15.0):
+    Ns, P, B, Q, M_L, x = oracle_sample(workload, G, budget_s / 2)
+    times = time_oracle(Ns, P, B, Q, M_L, x, budget_s / 2)
+    t = statistics.median(times)
+    return {"value": flops_fft(Ns) / t / 1e9, "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
+            "sample": f"oracle.fmmfft (numpy float64, 1 thread) at N={Ns} with P={P}, B={B}, Q={Q}, M_L={M_L}; "
+                      f"median of {len(times)} runs ({t:.3f} s each)"}
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle as it stands, on host cores, rank 0 only."""
+    if rank != 0:
+        return
+    workload = args.workload or ("cfg2" if world == 1 else "cfg3")
+    N, prec, Pf, B, Q, M_L, desc = WORKLOADS[workload]
+    per_step = max(0.05, 150.0 / (args.steps + args.warmup))
+    Ns, P, B, Q, M_L, x = oracle_sample(workload, world, per_step)
+    from oracle import fmmfft_oracle as O
+    try:
+        from threadpoolctl import threadpool_limits
+        lim = threadpool_limits(1)
+    except Exception:
+        lim = None
+    for _ in range(args.warmup):
+        O.fmmfft(x, P, B, Q, M_L)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        O.fmmfft(x, P, B, Q, M_L)
+        times.append(time.perf_counter() - t0)
+    del lim
+    t = sum(times) / len(times)
+    val = flops_fft(Ns) / t / 1e9
+    sample = (f"oracle.fmmfft (numpy float64, 1 thread) at N={Ns} (of N={N}) with P={P}, B={B}, Q={Q}, "
+              f"M_L={M_L}, one run per step")
+    line = {"impl": "reference", "metric": "1D C2C FFT GFLOP/s (5N log2N/t)", "value": val, "unit": "GFLOP/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": workload, "desc": desc, "N_sample": Ns},
+            "cpu_baseline": {"value": val, "unit": "GFLOP/s", "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": val, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------------------ GPU arm
+def run_fmmfft(args, rank, world, local_rank):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import synth_inputs as SI
+    from paper_conf_sc_cecka17_b200 import FmmFFT, init_comm
+    from paper_conf_sc_cecka17_b200 import build as b
+
+    if rank == 0:
+        b.build()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.set_device(local_rank)
+    if world > 1:
+        init_comm()
+    workload = args.workload or ("cfg2" if world == 1 else "cfg3")
+    N, prec, Pf, B, Q, M_L, desc = WORKLOADS[workload]
+    P = Pf(world)
+    G = world
+    npdt = np.complex64 if prec == "c64" else np.complex128
+    esz = 8 if prec == "c64" else 16
+    plan = FmmFFT(N=N, P=P, G=G, B=B, Q=Q, precision=prec, M_L=M_L, profile=True)
+    info = plan.info
+    x_host = SI.shard(N, G, rank, dtype=npdt)
+    x = torch.from_numpy(x_host).cuda()
+    y = torch.empty_like(x)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    stream = torch.cuda.current_stream()
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    for _ in range(max(3, args.warmup)):
+        flush.zero_()
+        plan(x, y)
+    torch.cuda.synchronize()
+
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    stage_sum = {}
+    sampler = ClockSampler(torch.cuda.current_device() if "CUDA_VISIBLE_DEVICES" not in os.environ else local_rank)
+    with sampler:
+        barrier()
+        torch.cuda.synchronize()
+        sampler.active.set()
+        for k in range(args.steps):
+            flush.zero_()
+            ev[k][0].record(stream)
+            plan(x, y, stream)
+            ev[k][1].record(stream)
+            st = plan.stage_times()           # syncs this step's events (after the step is enqueued)
+            for n_, v in st.items():
+                stage_sum[n_] = stage_sum.get(n_, 0.0) + v
+        torch.cuda.synchronize()
+        barrier()
+        sampler.active.clear()
+    step_ms = [a.elapsed_time(b_) for a, b_ in ev]
+    t_local = sum(step_ms) / len(step_ms)
+    t_max = torch.tensor([t_local], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
+    ms_per_step = float(t_max.item())
+    value = flops_fft(N) / (ms_per_step * 1e-3) / 1e9
+    stages = {n_: v / args.steps for n_, v in stage_sum.items()}
+
+    # ---- end to end through the C ABI with host buffers (H2D + execute + D2H per step)
+    xh = torch.from_numpy(x_host).pin_memory()
+    yh = torch.empty_like(xh).pin_memory()
+    plan_e2e = FmmFFT(N=N, P=P, G=G, B=B, Q=Q, precision=prec, M_L=M_L)
+    for _ in range(2):
+        plan_e2e.execute_host(xh, yh, stream)
+    torch.cuda.synchronize()
+    k_e2e = max(3, min(args.steps, 50))
+    ee = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(k_e2e)]
+    barrier()
+    torch.cuda.synchronize()
+    for k in range(k_e2e):
+        ee[k][0].record(stream)
+        plan_e2e.execute_host(xh, yh, stream)
+        ee[k][1].record(stream)
+    torch.cuda.synchronize()
+    barrier()
+    e2e_local = sum(a.elapsed_time(b_) for a, b_ in ee) / k_e2e
+    e2e_t = torch.tensor([e2e_local], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+    e2e_ms = float(e2e_t.item())
+    # correctness of the timed output on a sample (rank 0's block): Parseval over the whole job
+    ny = torch.sum(torch.abs(y.to(torch.complex128)) ** 2)
+    nx = torch.sum(torch.abs(x.to(torch.complex128)) ** 2)
+    if world > 1:
+        dist.all_reduce(ny)
+        dist.all_reduce(nx)
+    parseval = float(ny / (N * nx) - 1)
+
+    if rank != 0:
+        return
+    peaks = load_peaks()
+    fl = near_up_flops(N, P, B, Q, M_L, G)
+    t_near = stages.get("near_up", float("nan")) * 1e-3
+    sm_max = peaks.get("sm_max_mhz", 1965.0)
+    if prec == "c64":
+        peak = 148 * 128 * 2 * sm_max * 1e6 / 1e12            # FP32 FMA lanes x 2 flops x max clock
+    else:
+        peak = 148 * 64 * 2 * sm_max * 1e6 / 1e12             # FP64 FMA lanes (half rate)
+    achieved = fl / t_near / 1e12
+    clocks = sampler.summary()
+    line = {
+        "metric": "1D C2C FFT GFLOP/s (5N log2N/t)", "value": value, "unit": "GFLOP/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f32" if prec == "c64" else "f64",
+        "data": "synthetic",
+        "config": {"workload": workload, "desc": desc, "N": N, "P": P, "G": G, "B": B, "Q": Q, "M_L": M_L,
+                   "L": info["L"], "precision": prec, "l2": "flushed (256 MiB write between steps, outside events)",
+                   "parseval_rel_dev": parseval},
+        "roofline": {"kernel": "k_near_up (S2T + S2M)", "bound": "alu", "achieved": achieved, "peak": peak,
+                     "unit": "TFLOP/s", "frac": achieved / peak, "traffic": load_traffic(workload, G),
+                     "algorithmic_flops_per_launch": fl, "avg_launch_ms": t_near * 1e3,
+                     "peak_basis": f"148 SMs x {'128 FP32' if prec == 'c64' else '64 FP64'} FMA/clk x 2 x {sm_max} MHz"},
+        "stages_ms": stages,
+        "e2e": {"value": flops_fft(N) / (e2e_ms * 1e-3) / 1e9, "unit": "GFLOP/s",
+                "h2d_bytes_per_step": (N // G) * esz, "d2h_bytes_per_step": (N // G) * esz, "ms_per_step": e2e_ms},
+        "gpu_launches": info["kernels_per_execute"] * args.steps,
+        "clocks": {k: clocks[k] for k in ("sm_mhz", "sm_max_mhz", "reasons")},
+    }
+    if world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(workload, G)
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="fmmfft", choices=["fmmfft", "reference"])
+    ap.add_argument("--workload", default=None, choices=sorted(WORKLOADS))
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(3, args.warmup)
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        print(f"warning: --gpus {args.gpus} but WORLD_SIZE={world}; using WORLD_SIZE", file=sys.stderr)
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    try:
+        run_fmmfft(args, rank, world, local_rank)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.barrier()
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

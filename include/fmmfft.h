@@ -1,0 +1,145 @@
+/*
+ * fmmfft.h — C ABI of the B200-native FMM-FFT (Cecka, "Low Communication FMM-Accelerated FFT
+ * on GPUs", SC17). Citations "P:<lines>" point into the paper text.
+ *
+ * WHAT IS COMPUTED. The forward, unnormalised, in-order 1D complex DFT of length N,
+ *     y_k = sum_{j<N} x_j w_N^{jk},  w_N = exp(-2 pi i / N)            (eq. 1)
+ * by the FMM-FFT factorisation F_N = F_{M,P} H^_{M,P}, N = M P          (eq. 2):
+ * P-1 interleaved periodic 1D FMMs with the cotangent kernel (Algorithm 1),
+ * the POST scaling (line 15), and an M x P 2D FFT with ONE all-to-all transpose (line 16,
+ * P:389-399). The FMM uses Q Chebyshev nodes per box, M_L points per leaf box,
+ * leaf level L = log2(N / (P M_L)) and base level B (Table 1).
+ *
+ * DATA. Input and output are interleaved complex (float2 for FMMFFT_C64, double2 for
+ * FMMFFT_C128), block-distributed in natural order: rank g of G holds x[g N/G, (g+1) N/G)
+ * and receives y[g N/G, (g+1) N/G). For G = 1 these are the whole vectors.
+ *
+ * OWNERSHIP. The plan owns every workspace buffer (halos, tree, transpose buffers, operator
+ * tables) and, for G > 1, uses the communicator set up by fmmfft_comm_init. Caller-owned
+ * buffers are never retained after a call returns (execution is stream-ordered: they must stay
+ * valid until the stream reaches the end of the enqueued work).
+ *
+ * ERRORS. Every entry point returns an fmmfft_status_t; no C++ exception crosses the
+ * boundary. On failure fmmfft_last_error() returns a thread-local message. Invalid arguments
+ * return FMMFFT_INVALID_VALUE and leave outputs untouched.
+ *
+ * THREADING. A plan is not re-entrant: no concurrent execute on one plan. Different plans
+ * may be used from different threads.
+ */
+#ifndef FMMFFT_H
+#define FMMFFT_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define FMMFFT_API __attribute__((visibility("default")))
+#else
+#define FMMFFT_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct fmmfft_plan_s* fmmfft_plan_t;
+
+/* Arithmetic type. C64 = complex64 storage, fp32 arithmetic; C128 = complex128, fp64. */
+typedef enum { FMMFFT_C64 = 0, FMMFFT_C128 = 1 } fmmfft_precision_t;
+
+typedef enum {
+    FMMFFT_SUCCESS = 0,
+    FMMFFT_INVALID_VALUE = 1,   /* an argument violates the contract below                 */
+    FMMFFT_UNSUPPORTED = 2,     /* valid in the paper, not supported by this build / device */
+    FMMFFT_ALLOC_FAILED = 3,    /* device or host allocation failed                          */
+    FMMFFT_CUDA_ERROR = 4,      /* a CUDA runtime call or kernel launch failed               */
+    FMMFFT_NCCL_ERROR = 5,      /* NCCL missing or an NCCL call failed                       */
+    FMMFFT_NOT_INITIALIZED = 6  /* G > 1 without fmmfft_comm_init                            */
+} fmmfft_status_t;
+
+/* Plan flags (fmmfft_plan_ex). */
+#define FMMFFT_FLAG_VIRTUAL 1u  /* G "virtual ranks" in this process on the current device:
+                                   the distributed data flow (halos, all-gather, all-to-all)
+                                   runs with device-to-device copies instead of NCCL. in/out
+                                   are then the FULL length-N vectors. For testing the
+                                   partitioned algorithm on one GPU. */
+#define FMMFFT_FLAG_PROFILE 2u  /* record CUDA events around every stage (fmmfft_stage_times) */
+
+/* ---------------------------------------------------------------- communicator (G > 1)
+ * One process per GPU. Rank 0 calls fmmfft_get_unique_id and broadcasts the 128 bytes (e.g.
+ * through torch.distributed); every rank then calls fmmfft_comm_init with its rank, the
+ * world size G and that id. Binds the communicator to the CURRENT CUDA device. NCCL is loaded
+ * at run time (dlopen "libnccl.so.2"); FMMFFT_NCCL_ERROR if it cannot be found. */
+FMMFFT_API fmmfft_status_t fmmfft_get_unique_id(unsigned char id[128]);
+FMMFFT_API fmmfft_status_t fmmfft_comm_init(int rank, int G, const unsigned char id[128]);
+FMMFFT_API fmmfft_status_t fmmfft_comm_destroy(void);
+
+/* ---------------------------------------------------------------- plans
+ * fmmfft_plan: N = M P points, P FMMs interleaved (P - 1 non-trivial), G ranks, base level
+ * B, Q Chebyshev nodes, M_L = 64 (the paper's large-N leaf size).
+ * fmmfft_plan_ex: same with an explicit M_L and flags.
+ * Requirements (else FMMFFT_INVALID_VALUE):
+ *   N, P, M_L powers of two; P >= 2; G in {1, 2, 4, 8}; P % G == 0; N % (P M_L) == 0;
+ *   L = log2(N / (P M_L)) >= B >= 2; 2^L % G == 0; 2 <= Q <= 32;
+ *   16 <= M_L <= 256; P <= 2048; M = N / P >= 2 G.
+ *   Without FMMFFT_FLAG_VIRTUAL and G > 1, fmmfft_comm_init must have been called with the
+ *   same G (else FMMFFT_NOT_INITIALIZED). The device must be sm_100 (else UNSUPPORTED).
+ * Collective when G > 1 (non-virtual): every rank creates its plan with identical arguments.
+ * Allocates all device workspace and uploads the operator tables (computed in fp64 on the
+ * host: S2M/L2T, M2M/L2L P:630-800, S2T P:843-860, M2L P:902-947, rho_p P:374). */
+FMMFFT_API fmmfft_status_t fmmfft_plan(fmmfft_plan_t* plan, long long N, int P, int G, int B, int Q,
+                            fmmfft_precision_t precision);
+FMMFFT_API fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, int B, int Q,
+                               fmmfft_precision_t precision, int M_L, unsigned flags);
+
+/* Forward transform. in, out: device pointers on the plan's device, N/G complex elements
+ * each (N for a virtual plan), 16-byte aligned, non-overlapping (else INVALID_VALUE).
+ * in is not modified. Asynchronous on `stream` (a cudaStream_t; NULL = legacy default
+ * stream); no host synchronisation. Collective when G > 1. */
+FMMFFT_API fmmfft_status_t fmmfft_execute(fmmfft_plan_t plan, const void* in, void* out, void* stream);
+
+/* End-to-end variant with HOST buffers (pinned for full overlap; pageable works): copies
+ * in -> device, executes, copies the result -> out, all enqueued on `stream`. The caller
+ * synchronises the stream before reading out. */
+FMMFFT_API fmmfft_status_t fmmfft_execute_host(fmmfft_plan_t plan, const void* in_host, void* out_host,
+                                    void* stream);
+
+FMMFFT_API fmmfft_status_t fmmfft_destroy(fmmfft_plan_t plan);
+
+/* ---------------------------------------------------------------- introspection */
+typedef struct {
+    long long N;
+    int P, G, B, Q, M_L, L, precision;
+    long long M;            /* N / P                                               */
+    int level_gather;       /* l_g = max(B, log2 G + 1): finest all-gathered level (R16) */
+    int n_stages;           /* entries reported by fmmfft_stage_times               */
+    size_t workspace_bytes; /* device bytes owned by the plan (all virtual ranks)   */
+    int kernels_per_execute;/* this library's kernel launches per execute (per rank) */
+} fmmfft_info_t;
+
+FMMFFT_API fmmfft_status_t fmmfft_get_info(fmmfft_plan_t plan, fmmfft_info_t* info);
+
+/* Per-stage device times (ms) of the LAST execute of a plan created with
+ * FMMFFT_FLAG_PROFILE (else INVALID_VALUE); synchronises that execute's stream. Stage i's
+ * name is fmmfft_stage_name(i). n = capacity of ms[]; returns the count in *n_out. */
+FMMFFT_API fmmfft_status_t fmmfft_stage_times(fmmfft_plan_t plan, float* ms, int n, int* n_out);
+FMMFFT_API const char* fmmfft_stage_name(int i);
+
+/* Internal buffers after an execute, for stage-by-stage parity tests. `which`:
+ *   0 = T_near  [b][m][p]  (S2T output, N/G complex)
+ *   1 = M^l     [b][q][p]  (multipoles of level `level`, own boxes; slot p = FMM p)
+ *   2 = L^l     [b][q][p]  (local expansions of level `level`, own boxes)
+ *   3 = W       [k2][m]    (P-point FFT output before the transpose, N/G complex)
+ *   4 = r       [p]        (reductions r_p, slot p = FMM p; P complex)
+ * Returns a device pointer and its size in bytes; rank selects the virtual rank. */
+FMMFFT_API fmmfft_status_t fmmfft_debug_buffer(fmmfft_plan_t plan, int rank, int which, int level,
+                                    const void** ptr, size_t* bytes);
+
+/* Thread-local message of the last failure in this thread ("" if none). */
+FMMFFT_API const char* fmmfft_last_error(void);
+FMMFFT_API const char* fmmfft_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FMMFFT_H */

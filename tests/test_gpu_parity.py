@@ -1,0 +1,213 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU float64 oracle on the same seeded
+inputs — stage by stage (T_near, M^l, L^l, r, W) and end to end — plus edge cases.
+
+Tolerances: the north star's relative l2 bounds against the float64
+DFT of the same (rounded) input, 1e-5 for complex64 and 1e-11 for complex128; stage buffers
+against the oracle's same stage at 1e-5 (fp32 arithmetic over <= 3 M_L-term sums of
+cotangents) and 1e-12 (fp64).
+"""
+import numpy as np
+import pytest
+
+import synth_inputs as SI
+from oracle import distributed as D
+from oracle import fmmfft_oracle as O
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+TOL_E2E = {"c64": 1e-5, "c128": 1e-11}
+TOL_STAGE = {"c64": 1e-5, "c128": 1e-12}
+NPDT = {"c64": np.complex64, "c128": np.complex128}
+
+
+@pytest.fixture(scope="module")
+def F():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sc_cecka17_b200 import build
+    build.build()
+    from paper_conf_sc_cecka17_b200 import FmmFFT
+    return FmmFFT
+
+
+def run(F, N, P, B, Q, prec, M_L=64, G=1, virtual=False, seed=SI.DEFAULT_SEED):
+    x = SI.complex_uniform(0, N, seed=seed, dtype=NPDT[prec])
+    plan = F(N=N, P=P, G=G, B=B, Q=Q, precision=prec, M_L=M_L, virtual=virtual)
+    xd = torch.from_numpy(x).cuda()
+    y = plan(xd)
+    torch.cuda.synchronize()
+    return plan, x, y.cpu().numpy()
+
+
+def rel(a, b):
+    return O.rel_l2(np.asarray(a, dtype=np.complex128), b)
+
+
+# ------------------------------------------------------------------ end to end
+@pytest.mark.parametrize("N,P,B,Q,prec,M_L", [
+    (1 << 12, 16, 2, 16, "c128", 64),      # cfg1 (L = B = 2)
+    (1 << 12, 16, 2, 16, "c64", 64),
+    (1 << 12, 16, 2, 16, "c128", 16),      # cfg1 with L = 4
+    (1 << 20, 64, 2, 16, "c64", 64),       # cfg2 (the bench workload at N = 1)
+    (1 << 20, 64, 2, 16, "c128", 64),
+    (1 << 16, 32, 3, 16, "c64", 32),
+    (1 << 16, 8, 4, 16, "c128", 16),
+    (1 << 18, 128, 2, 24, "c128", 64),     # Q = 24 (cfg4's order)
+    (1 << 18, 256, 2, 8, "c64", 16),       # Q = 8 (the paper's single-precision order)
+    (1 << 17, 2, 3, 16, "c64", 128),       # P = 2, M_L = 128
+    (1 << 19, 512, 2, 16, "c64", 16),      # P = 512 (cfg4's P/G shape)
+    (1 << 16, 4, 5, 16, "c64", 32),
+])
+def test_end_to_end_vs_dft(F, N, P, B, Q, prec, M_L):
+    plan, x, y = run(F, N, P, B, Q, prec, M_L)
+    ref = O.dft_direct(x) if N <= 1 << 12 else O.fft_radix2(x)
+    err = rel(y, ref)
+    tol = TOL_E2E[prec] if Q >= 16 else 1e-4
+    if prec == "c128" and Q >= 16:
+        tol = max(tol, 0)  # 1e-11
+    assert err < tol, err
+    if prec == "c128" and Q >= 16:
+        # the FMM itself reaches the paper's double-precision accuracy
+        assert err < (2e-14 if M_L >= 32 else 3e-14) * 4
+
+
+def test_cfg1_c128_matches_oracle_and_direct_dft(F):
+    plan, x, y = run(F, 1 << 12, 16, 2, 16, "c128")
+    assert rel(y, O.fmmfft(x, 16, 2, 16)) < 1e-13
+    assert rel(y, O.dft_direct(x)) < 1e-11
+
+
+# ------------------------------------------------------------------ stage by stage
+@pytest.mark.parametrize("prec", ["c64", "c128"])
+@pytest.mark.parametrize("N,P,B,Q,M_L", [(1 << 16, 16, 2, 16, 32), (1 << 18, 64, 3, 16, 64)])
+def test_stages_match_oracle(F, prec, N, P, B, Q, M_L):
+    plan, x, y = run(F, N, P, B, Q, prec, M_L)
+    L = O.tree_levels(N, P, M_L)
+    S = x.astype(np.complex128).reshape(2 ** L, M_L, P)
+    st = O.fmm_stages(S, N, P, B, Q)
+    tol = TOL_STAGE[prec]
+    Tn = plan.debug_buffer("T_near").cpu().numpy().reshape(2 ** L, M_L, P)
+    assert rel(Tn, st["T_near"]) < tol
+    assert np.array_equal(Tn[:, :, 0], S[:, :, 0].astype(Tn.dtype))        # p = 0 copies exactly
+    for lev in range(B, L + 1):
+        Mg = plan.debug_buffer("M", lev).cpu().numpy().reshape(2 ** lev, Q, P)
+        assert rel(Mg[:, :, 1:], st["M"][lev]) < tol, ("M", lev)
+        Lg = plan.debug_buffer("L", lev).cpu().numpy().reshape(2 ** lev, Q, P)
+        assert rel(Lg[:, :, 1:], st["L"][lev]) < tol, ("L", lev)
+    r = plan.debug_buffer("r").cpu().numpy()
+    assert rel(r[1:], st["r"]) < tol
+    # W = P-point FFTs of POST(T) (before the transpose), stored [k2][m]
+    T = O.post(st["T"], st["r"], N, P).reshape(N // P, P)
+    W = O.fft_radix2(T, axis=1).T
+    Wg = plan.debug_buffer("W").cpu().numpy().reshape(P, N // P)
+    assert rel(Wg, W) < tol
+    assert rel(y, O.fft2d_MP(O.post(st["T"], st["r"], N, P).reshape(N), N // P, P)) < tol
+
+
+# ------------------------------------------------------------------ distributed data flow (virtual ranks)
+@pytest.mark.parametrize("N,P,B,Q,prec,M_L,G", [
+    (1 << 14, 16, 2, 16, "c64", 16, 2),
+    (1 << 16, 32, 2, 16, "c128", 16, 4),
+    (1 << 16, 32, 2, 16, "c64", 16, 8),      # l_g = 4 > B: replicated top levels
+    (1 << 18, 64, 4, 16, "c64", 32, 8),      # l_g = B = 4
+    (1 << 16, 16, 2, 16, "c128", 64, 8),     # L = 6, l_g = 4
+    (1 << 15, 16, 2, 16, "c64", 64, 8),      # L = 5: one box per rank at level 3
+    (1 << 20, 128, 2, 24, "c128", 64, 8),    # cfg4 shape, reduced N
+])
+def test_virtual_ranks_vs_oracle(F, N, P, B, Q, prec, M_L, G):
+    plan, x, y = run(F, N, P, B, Q, prec, M_L, G=G, virtual=True)
+    ref = O.fft_radix2(x)
+    assert rel(y, ref) < TOL_E2E[prec]
+    assert rel(y, D.fmmfft_virtual(x.astype(np.complex128), P, B, Q, M_L, G)) < (TOL_E2E[prec] if prec == "c64" else 1e-12)
+
+
+def test_virtual_matches_single_rank(F):
+    N, P, B, Q, M_L = 1 << 18, 64, 2, 16, 32
+    _, x, y1 = run(F, N, P, B, Q, "c128", M_L, G=1)
+    _, _, y8 = run(F, N, P, B, Q, "c128", M_L, G=8, virtual=True)
+    assert rel(y8, y1) < 1e-13
+
+
+# ------------------------------------------------------------------ structured inputs, edge cases
+def test_delta_and_tone(F):
+    N, P = 1 << 16, 32
+    plan = F(N=N, P=P, B=2, Q=16, precision="c128")
+    k = np.arange(N)
+    y = plan(torch.from_numpy(SI.delta(N, 12345)).cuda()).cpu().numpy()
+    assert np.max(np.abs(y - np.exp(-2j * np.pi * ((12345 * k) % N) / N))) < 1e-12
+    y = plan(torch.from_numpy(SI.tone(N, 999)).cuda()).cpu().numpy()
+    e = np.zeros(N, complex)
+    e[999] = N
+    assert np.max(np.abs(y - e)) < 1e-9 * N
+    y = plan(torch.zeros(N, dtype=torch.complex128, device="cuda")).cpu().numpy()
+    assert np.all(y == 0)
+
+
+def test_input_not_modified_and_repeatable(F):
+    N, P = 1 << 16, 16
+    plan = F(N=N, P=P, B=2, Q=16, precision="c64")
+    x = torch.from_numpy(SI.complex_uniform(0, N, dtype=np.complex64)).cuda()
+    x0 = x.clone()
+    y1 = plan(x)
+    y2 = plan(x)
+    torch.cuda.synchronize()
+    assert torch.equal(x, x0)
+    assert torch.equal(y1, y2)                 # deterministic: no atomics on the path
+
+
+def test_execute_rejects_bad_buffers(F):
+    from paper_conf_sc_cecka17_b200._lib import FmmfftError
+    N = 1 << 16
+    plan = F(N=N, P=16, B=2, Q=16, precision="c64")
+    x = torch.zeros(N, dtype=torch.complex64, device="cuda")
+    with pytest.raises(FmmfftError):
+        plan(x, out=x)                           # in == out overlap
+    with pytest.raises(ValueError):
+        plan(torch.zeros(N, dtype=torch.complex128, device="cuda"))
+
+
+def test_execute_host_path(F):
+    N, P = 1 << 18, 64
+    plan = F(N=N, P=P, B=2, Q=16, precision="c64")
+    x = SI.complex_uniform(0, N, dtype=np.complex64)
+    xh = torch.from_numpy(x).pin_memory()
+    yh = torch.empty_like(xh).pin_memory()
+    s = torch.cuda.current_stream()
+    plan.execute_host(xh, yh, s)
+    s.synchronize()
+    assert rel(yh.numpy(), O.fft_radix2(x)) < 1e-5
+
+
+def test_profile_stage_times(F):
+    plan = F(N=1 << 20, P=64, B=2, Q=16, precision="c64", profile=True)
+    x = torch.from_numpy(SI.complex_uniform(0, 1 << 20, dtype=np.complex64)).cuda()
+    plan(x)
+    t = plan.stage_times()
+    assert list(t) == ["comm_S", "near_up", "m2m", "comm_M", "top", "down", "post_pfft", "a2a", "mfft"]
+    assert all(v >= 0 for v in t.values()) and t["near_up"] > 0
+    assert plan.info["kernels_per_execute"] > 5
+
+
+# ------------------------------------------------------------------ full-size bench configs, sampled
+def sampled_dft(x, ks):
+    N = len(x)
+    j = np.arange(N, dtype=np.int64)
+    xc = x.astype(np.complex128)
+    return np.array([np.dot(xc, np.exp(-2j * np.pi * ((j * k) % N) / N)) for k in ks])
+
+
+@pytest.mark.parametrize("N,P,B,Q,prec,G", [
+    (1 << 20, 64, 2, 16, "c64", 1),      # cfg2 — exactly the bench.py N=1 launch configuration
+    (1 << 26, 128, 4, 16, "c64", 8),     # cfg3 shape (G = 8) as virtual ranks on one GPU
+])
+def test_full_size_sampled(F, N, P, B, Q, prec, G):
+    plan, x, y = run(F, N, P, B, Q, prec, 64, G=G, virtual=G > 1)
+    rng = np.random.default_rng(0)
+    ks = np.concatenate([[0, 1, N // 2, N - 1], rng.integers(0, N, 8)])
+    ref = sampled_dft(x, ks)
+    assert np.linalg.norm(y[ks] - ref) / np.linalg.norm(ref) < 1e-5
+    # Parseval holds at any size: ||y||^2 = N ||x||^2
+    ny = np.sum(np.abs(y.astype(np.complex128)) ** 2)
+    nx = np.sum(np.abs(x.astype(np.complex128)) ** 2)
+    assert abs(ny / (N * nx) - 1) < 1e-5
