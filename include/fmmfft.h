@@ -114,7 +114,7 @@ typedef struct {
     int level_gather;       /* l_g = max(B, log2 G + 1): finest all-gathered level (R16) */
     int n_stages;           /* entries reported by fmmfft_stage_times               */
     size_t workspace_bytes; /* device bytes owned by the plan (all virtual ranks)   */
-    int kernels_per_execute;/* this library's kernel launches per execute (per rank) */
+    int kernels_per_execute;/* kernels this library launched in the last execute (0 before) */
 } fmmfft_info_t;
 
 FMMFFT_API fmmfft_status_t fmmfft_get_info(fmmfft_plan_t plan, fmmfft_info_t* info);

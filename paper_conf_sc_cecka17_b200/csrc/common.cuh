@@ -54,4 +54,22 @@ template <> __device__ __forceinline__ double2 twiddle<double>(long long num, lo
 __device__ __forceinline__ float2 ldg_c(const float2* p) { return __ldg(p); }
 __device__ __forceinline__ double2 ldg_c(const double2* p) { return __ldg(p); }
 
+// cp.async (LDGSTS): global -> shared without a register round trip, so a thread can have many
+// copies in flight; cp_async_wait_all() + __syncthreads() publishes them.
+template <int BYTES>
+__device__ __forceinline__ void cp_async(void* smem, const void* gmem) {
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+    if constexpr (BYTES == 16)
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(sa), "l"(gmem) : "memory");
+    else
+        asm volatile("cp.async.ca.shared.global [%0], [%1], %2;\n" ::"r"(sa), "l"(gmem), "n"(BYTES) : "memory");
+}
+template <typename T>
+__device__ __forceinline__ void cp_async_elem(T* smem, const T* gmem) { cp_async<sizeof(T)>(smem, gmem); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+template <int N> __device__ __forceinline__ void cp_async_wait_group() {
+    asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory");
+}
+
 }  // namespace fmmfft

@@ -7,22 +7,28 @@
 //
 //   comm_S    S halo (line 2)                          NCCL send/recv | D2D | none (G = 1)
 //   near_up   S2T + S2M (lines 1, 3)                   k_near_up
-//   m2m       M2M for l = L-1 .. l_g (line 5)          k_m2m per level
+//   m2m       M2M for l = L-1 .. l_g (line 5)          k_up (up to 4 levels per launch)
 //   comm_M    M^l halos for l > l_g (line 7) + all-gather of level l_g (line 9, reading R16)
-//   top       M2M l_g-1 .. B on the gathered level, M2L-B (line 10), REDUCE (line 11),
+//   top       M2M l_g-1 .. B on the gathered level, M2L-B (line 10) + REDUCE (line 11),
 //             M2L + L2L for B < l <= l_g (replicated top of the tree)
 //   down      M2L-l (line 8) + L2L (line 13) for l = l_g+1 .. L   k_down per level
 //   post_pfft L2T + POST + P-point FFTs + transposed store (lines 14-16)
 //   a2a       the one all-to-all transpose (line 16)
 //   mfft      P/G M-point FFTs, multi-pass Stockham (line 16)
+//
+// The whole sequence is captured once per (in, out) pair into a CUDA graph (on a plan-owned
+// stream) and replayed on the caller's stream: one launch per execute instead of ~20.
 #include <cuda_runtime.h>
 
 #include <algorithm>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <string>
+#include <type_traits>
 #include <vector>
 
 #include "../../include/fmmfft.h"
@@ -61,7 +67,15 @@ static fmmfft_status_t fail(fmmfft_status_t st, const char* fmt, ...) {
             return fail(FMMFFT_NCCL_ERROR, "%s failed: %s", #expr, nccl().GetErrorString(r_));  \
     } while (0)
 
-#define LAUNCH_CHECK() CUDA_TRY(cudaGetLastError())
+#define LAUNCH_CHECK() do { ++nlaunch; CUDA_TRY(cudaGetLastError()); } while (0)
+
+// compile-time dispatch of a runtime value onto a list of template values
+template <int... Vs, typename F>
+static bool dispatch(int v, F&& f) {
+    bool hit = false;
+    ((v == Vs ? (f(std::integral_constant<int, Vs>{}), hit = true) : false), ...);
+    return hit;
+}
 
 // ------------------------------------------------------------------ communicator
 struct Comm {
@@ -104,6 +118,13 @@ struct RankBufs {
     std::vector<void*> Mpad, Lloc, Mfull, Lfull;   // indexed by level
 };
 
+struct GraphEntry {
+    const void* in = nullptr;
+    void* out = nullptr;
+    cudaGraphExec_t exec = nullptr;
+    int nlaunch = 0;
+};
+
 }  // namespace fmmfft
 
 struct fmmfft_plan_s {
@@ -114,6 +135,8 @@ struct fmmfft_plan_s {
     bool virt = false;
     int device = -1;
     size_t esz = 0, rsz = 0;
+    int PCn = 0, PCd = 0;            // p-chunks of near_up and of the tree kernels
+    int s2t_chunk = 0, m2l_chunk = 0, m2lB_chunk = 0;   // table chunk strides (elements)
     // device tables
     void* s2m = nullptr;
     void* m2m = nullptr;
@@ -121,13 +144,17 @@ struct fmmfft_plan_s {
     void* rho = nullptr;
     void* m2lB = nullptr;
     std::vector<void*> m2l;          // by level
+    std::vector<void*> m2l_pmaj;     // p-major copies for the fused per-p tree (G = 1), by level
+    bool tree_p = false;             // use k_tree_p for the far field
     std::vector<fmmfft::RankBufs> ranks;
     std::vector<int> radices;        // M-FFT passes
     size_t ws_bytes = 0;
     int kernels = 0;
     cudaEvent_t ev[fmmfft::ST_COUNT + 1] = {};
-    cudaStream_t last_stream = nullptr;
     bool have_times = false;
+    bool use_graph = true;
+    cudaStream_t cap_stream = nullptr;
+    std::vector<fmmfft::GraphEntry> graphs;
     std::vector<void*> allocs;
 };
 
@@ -135,6 +162,7 @@ namespace fmmfft {
 
 static fmmfft_status_t dalloc(fmmfft_plan_s* p, void** ptr, size_t bytes) {
     if (bytes == 0) bytes = 16;
+    bytes = (bytes + 255) & ~(size_t)255;
     cudaError_t e = cudaMalloc(ptr, bytes);
     if (e != cudaSuccess) return fail(FMMFFT_ALLOC_FAILED, "cudaMalloc(%zu) failed: %s", bytes, cudaGetErrorString(e));
     p->allocs.push_back(*ptr);
@@ -154,6 +182,7 @@ static fmmfft_status_t upload(fmmfft_plan_s* p, void** dst, const std::vector<do
 
 static int ilog2(long long v) { int l = 0; while ((1LL << l) < v) ++l; return l; }
 static bool pow2(long long v) { return v > 0 && (v & (v - 1)) == 0; }
+static int pad16(int elems, int esz) { return ((elems * esz + 15) / 16) * 16 / esz; }
 
 template <typename R>
 static fmmfft_status_t build_tables(fmmfft_plan_s* p) {
@@ -172,32 +201,49 @@ static fmmfft_status_t build_tables(fmmfft_plan_s* p) {
         for (int k = 0; k < 2 * Q; ++k)
             m2m[(size_t)q * 2 * Q + k] = lagr(z, q, (z[k % Q] + (k < Q ? -1.0 : 1.0)) / 2.0);
     if ((st = upload<R>(p, &p->m2m, m2m))) return st;
-    // S2T_{pk} = cot(pi (p + P k)/N), p > 0; delta_{k0} for p = 0, layout [k][p]
-    const int nK = 4 * M_L - 1;
-    std::vector<double> s2t((size_t)nK * P, 0.0);
-    for (int ki = 0; ki < nK; ++ki) {
-        const long long k = ki - (2 * M_L - 1);
-        for (int pp = 0; pp < P; ++pp)
-            s2t[(size_t)ki * P + pp] = pp == 0 ? (k == 0 ? 1.0 : 0.0) : cotpi((double)(pp + (long long)P * k) / (double)N);
-    }
+    // S2T_{pk} = cot(pi (p + P k)/N), p > 0; delta_{k0} for p = 0,
+    // layout [chunk][k][pl] for near_up's p-chunk PCn
+    const int nK = 4 * M_L - 1, PCn = p->PCn;
+    p->s2t_chunk = pad16(nK * PCn, sizeof(R));
+    std::vector<double> s2t((size_t)(P / PCn) * p->s2t_chunk, 0.0);
+    for (int pp = 0; pp < P; ++pp)
+        for (int ki = 0; ki < nK; ++ki) {
+            const long long k = ki - (2 * M_L - 1);
+            s2t[(size_t)(pp / PCn) * p->s2t_chunk + (size_t)ki * PCn + pp % PCn] =
+                pp == 0 ? (k == 0 ? 1.0 : 0.0) : cotpi((double)(pp + (long long)P * k) / (double)N);
+        }
     if ((st = upload<R>(p, &p->s2t, s2t))) return st;
     // M2L^l_{pijs} = cot(pi/2^l (z_j/2 - z_i/2 + s) + pi p/N) for FMM p (slot = p),
-    // layout [s][i][j][p]; s in {-3, -2, 2, 3} for l > B, and 2..2^B-2 at the base
+    // layout [chunk][s][i][j][pl]; s in {-3, -2, 2, 3} for l > B, 2..2^B-2 at the base
+    const int PCd = p->PCd;
     p->m2l.assign(p->L + 1, nullptr);
+    p->m2l_pmaj.assign(p->L + 1, nullptr);
     const int shifts[4] = {-3, -2, 2, 3};
     for (int lev = p->B; lev <= p->L; ++lev) {
         const bool base = lev == p->B;
         const int ns = base ? (1 << p->B) - 3 : 4;
-        std::vector<double> t((size_t)ns * Q * Q * P, 0.0);
+        const int chunk = pad16(ns * Q * Q * PCd, sizeof(R));
+        (base ? p->m2lB_chunk : p->m2l_chunk) = chunk;
+        std::vector<double> t((size_t)(P / PCd) * chunk, 0.0);
         for (int si = 0; si < ns; ++si) {
             const int s = base ? 2 + si : shifts[si];
             for (int i = 0; i < Q; ++i)
                 for (int j = 0; j < Q; ++j)
                     for (int pp = 1; pp < P; ++pp)
-                        t[(((size_t)si * Q + i) * Q + j) * P + pp] =
+                        t[(size_t)(pp / PCd) * chunk + (((size_t)si * Q + i) * Q + j) * PCd + pp % PCd] =
                             cotpi((z[j] / 2 - z[i] / 2 + s) / (double)(1LL << lev) + (double)pp / (double)N);
         }
         if ((st = upload<R>(p, base ? &p->m2lB : &p->m2l[lev], t))) return st;
+        if (p->tree_p) {                                   // [p][s][j][i] (i fastest) for k_tree_p
+            std::vector<double> tp((size_t)P * ns * Q * Q, 0.0);
+            for (int pp = 0; pp < P; ++pp)
+                for (int si = 0; si < ns; ++si)
+                    for (int i = 0; i < Q; ++i)
+                        for (int j = 0; j < Q; ++j)
+                            tp[(size_t)pp * ns * Q * Q + ((size_t)si * Q + j) * Q + i] =
+                                t[(size_t)(pp / PCd) * chunk + (((size_t)si * Q + i) * Q + j) * PCd + pp % PCd];
+            if ((st = upload<R>(p, &p->m2l_pmaj[lev], tp))) return st;
+        }
     }
     // rho_p = exp(-i pi p/P) sin(pi p/P) / M, interleaved complex; rho_0 unused
     std::vector<double> rho(2 * (size_t)P);
@@ -259,22 +305,73 @@ static fmmfft_status_t alloc_rank(fmmfft_plan_s* p, RankBufs& rb) {
 }
 
 static void destroy_plan(fmmfft_plan_s* p) {
+    for (auto& g : p->graphs)
+        if (g.exec) cudaGraphExecDestroy(g.exec);
     for (void* a : p->allocs) cudaFree(a);
     for (auto& ev : p->ev)
         if (ev) cudaEventDestroy(ev);
+    if (p->cap_stream) cudaStreamDestroy(p->cap_stream);
     delete p;
 }
 
-static int count_kernels(const fmmfft_plan_s* p) {
-    int k = 1;                          // near_up
-    k += p->L - p->lg;                  // m2m (distributed levels)
-    k += p->lg - p->B;                  // m2m on the gathered top
-    k += 2;                             // base M2L + reduce
-    k += p->lg - p->B;                  // replicated down levels
-    k += p->L - p->lg;                  // distributed down levels
-    k += 1;                             // post_pfft
-    k += (int)p->radices.size();        // M-FFT passes
-    return k * (p->virt ? p->G : 1);
+// Raise every kernel's dynamic shared memory cap once per process (not legal during capture).
+template <typename R>
+static fmmfft_status_t init_kernel_attrs() {
+    static std::once_flag once;
+    static cudaError_t err = cudaSuccess;
+    std::call_once(once, [] {
+        int dev = 0, optin = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+        auto set = [&](const void* f) {
+            cudaFuncAttributes fa;
+            cudaError_t e = cudaFuncGetAttributes(&fa, f);
+            if (e == cudaSuccess)
+                e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, optin - (int)fa.sharedSizeBytes);
+            if (e != cudaSuccess && err == cudaSuccess) err = e;
+        };
+        constexpr int IB = sizeof(R) == 4 ? 16 : 8;
+        auto per_pc = [&](auto pc) {
+            constexpr int PCv = decltype(pc)::value;
+            set((const void*)k_near_up<R, IB, PCv>);
+            if constexpr (PCv <= (sizeof(R) == 4 ? 16 : 8)) {
+                set((const void*)k_up<R, PCv>);
+                set((const void*)k_down<R, 2, PCv>);
+                set((const void*)k_down<R, 4, PCv>);
+                set((const void*)k_down<R, 8, PCv>);
+                set((const void*)k_down<R, 16, PCv>);
+                set((const void*)k_base<R, 4, PCv>);
+                set((const void*)k_base<R, 8, PCv>);
+                set((const void*)k_base<R, 16, PCv>);
+                set((const void*)k_base<R, 32, PCv>);
+                set((const void*)k_tree_down<R, PCv, 1>);
+                set((const void*)k_tree_down<R, PCv, 2>);
+                set((const void*)k_tree_down<R, PCv, 4>);
+                set((const void*)k_tree_down<R, PCv, 8>);
+                set((const void*)k_tree_down<R, PCv, 16>);
+            }
+        };
+        for (int pc = 2; pc <= (sizeof(R) == 4 ? 32 : 16); pc *= 2) dispatch<2, 4, 8, 16, 32>(pc, per_pc);
+        set((const void*)k_tree_p<R, 1>);
+        set((const void*)k_tree_p<R, 2>);
+        set((const void*)k_tree_p<R, 4>);
+        set((const void*)k_tree_p<R, 8>);
+        for (int lp = 1; lp <= 11; ++lp)
+            dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 11>(lp, [&](auto v) { set((const void*)k_post_pfft<R, decltype(v)::value>); });
+        for (int lr = 1; lr <= 10; ++lr)
+            dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10>(lr, [&](auto v) { set((const void*)k_fft_pass<R, decltype(v)::value>); });
+    });
+    CUDA_TRY(err);
+    return FMMFFT_SUCCESS;
+}
+
+// shared memory of k_tree_p: the multipole pyramid + M2M + all M2L tables of one FMM
+static size_t tree_p_smem(const fmmfft_plan_s* p, int threads) {
+    (void)threads;
+    const size_t Q = p->Q;
+    const size_t npyr = (((size_t)2 << p->L) - ((size_t)1 << p->B)) * Q;
+    const size_t tabs = ((size_t)(1 << p->B) - 3) * Q * Q + (size_t)(p->L - p->B) * 4 * Q * Q;
+    return npyr * p->esz + (4 * Q * Q + tabs) * p->rsz + 32 * p->esz;
 }
 
 // ------------------------------------------------------------------ execute
@@ -285,18 +382,26 @@ struct Exec {
     cudaStream_t s;
     std::vector<const C*> in;    // per rank
     std::vector<C*> out;
+    int nlaunch = 0;             // kernels launched by this execute (all virtual ranks)
 
     static constexpr int IB = sizeof(R) == 4 ? 16 : 8;
-    static constexpr int EPT = sizeof(R) == 4 ? 32 : 16;
     static constexpr int TILE = sizeof(R) == 4 ? kTileF : kTileD;
-    int PC() const { return std::min(p->P, sizeof(R) == 4 ? 32 : 16); }
     size_t QP() const { return (size_t)p->Q * p->P; }
     int nb_at(int lev) const { return (int)((1LL << lev) / p->G); }
     C* interior(void* pad) const { return (C*)pad + 2 * QP(); }
     ncclDataType_t nt() const { return sizeof(R) == 4 ? ncclFloat : ncclDouble; }
+    int grank(const RankBufs& rb) const { return p->virt ? rb.g : (p->G > 1 ? g_comm.rank : 0); }
 
+    template <typename F> bool with_pcd(F&& f) const {
+        if constexpr (sizeof(R) == 4) return dispatch<2, 4, 8, 16>(p->PCd, f);
+        else return dispatch<2, 4, 8>(p->PCd, f);
+    }
+
+    // stage boundary event; inside a graph capture it must be an "external" record to become a
+    // real event-record node (a plain record during capture only expresses a dependency)
     fmmfft_status_t mark(int stage) {
-        if (p->flags & FMMFFT_FLAG_PROFILE) CUDA_TRY(cudaEventRecord(p->ev[stage], s));
+        if (p->flags & FMMFFT_FLAG_PROFILE)
+            CUDA_TRY(cudaEventRecordWithFlags(p->ev[stage], s, p->use_graph ? cudaEventRecordExternal : cudaEventRecordDefault));
         return FMMFFT_SUCCESS;
     }
 
@@ -329,44 +434,93 @@ struct Exec {
 
     // ---- near_up: S2T + S2M
     fmmfft_status_t near_up() {
-        const int PC_ = PC(), nib = p->M_L / IB;
+        const int PC_ = p->PCn, nib = p->M_L / IB;
         const int threads = PC_ * nib;
         const int npc = p->P / PC_;
         const int target = 2 * 148 * 2;
         const int bpc = std::max(1, (int)((long long)p->nb * npc / target));
         const dim3 grid((p->nb + bpc - 1) / bpc, npc);
-        const size_t smem = (size_t)3 * p->M_L * PC_ * sizeof(C) + (size_t)(4 * p->M_L - 1) * PC_ * sizeof(R) +
+        const size_t smem = (size_t)4 * p->M_L * PC_ * sizeof(C) + (size_t)p->s2t_chunk * sizeof(R) +
                             (size_t)p->Q * p->M_L * sizeof(R);
-        CUDA_TRY(cudaFuncSetAttribute(k_near_up<R, IB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         for (RankBufs& rb : p->ranks) {
             const C* S = in[p->virt ? rb.g : 0];
             const size_t box = (size_t)p->M_L * p->P;
             const C* hl = p->G == 1 ? S + (size_t)(p->nb - 1) * box : (const C*)rb.haloL;
             const C* hr = p->G == 1 ? S : (const C*)rb.haloR;
-            k_near_up<R, IB><<<grid, threads, smem, s>>>(S, hl, hr, (C*)rb.Tn, interior(rb.Mpad[p->L]),
-                                                       (const R*)p->s2t, (const R*)p->s2m, p->P, p->M_L,
-                                                       p->Q, p->nb, bpc, PC_);
+            auto go = [&](auto pc) {
+                constexpr int PCv = decltype(pc)::value;
+                if constexpr (sizeof(R) == 8 && PCv > 16) return;
+                else
+                    k_near_up<R, IB, PCv><<<grid, threads, smem, s>>>(S, hl, hr, (C*)rb.Tn, interior(rb.Mpad[p->L]),
+                                                                      (const R*)p->s2t, p->s2t_chunk, (const R*)p->s2m,
+                                                                      p->P, p->M_L, p->Q, p->nb, bpc);
+            };
+            dispatch<2, 4, 8, 16, 32>(PC_, go);
             LAUNCH_CHECK();
         }
         return FMMFFT_SUCCESS;
     }
 
-    fmmfft_status_t launch_m2m(const C* inl, C* outl, int nb_out) {
-        const long long total = (long long)nb_out * QP();
-        const int threads = 256;
-        const int blocks = (int)std::min<long long>((total + threads - 1) / threads, 148LL * 16);
-        const size_t smem = (size_t)2 * p->Q * p->Q * sizeof(R);
-        k_m2m<R><<<blocks, threads, smem, s>>>(inl, outl, (const R*)p->m2m, p->P, p->Q, nb_out);
-        LAUNCH_CHECK();
+    // M2M for levels from..to (from > to) starting at `inl` (level `from`, nb_from boxes),
+    // writing level l to outs(l); k_up handles up to 4 levels per launch.
+    template <typename OutF>
+    fmmfft_status_t launch_up(const C* inl, int from, int to, long long nb_from, OutF outs) {
+        const int PC_ = p->PCd;
+        int cur = from;
+        const C* src = inl;
+        long long nbc = nb_from;
+        while (cur > to) {
+            int h = std::min(4, cur - to);
+            while ((1LL << h) > nbc) --h;
+            UpOut uo{};
+            for (int l = 1; l <= h; ++l) uo.lev[l - 1] = outs(cur - l);
+            const size_t smem = ((size_t)1 << h) * p->Q * PC_ * sizeof(C) + (size_t)2 * p->Q * p->Q * sizeof(R);
+            const dim3 grid((unsigned)(nbc >> h), (unsigned)(p->P / PC_));
+            with_pcd([&](auto pc) {
+                constexpr int PCv = decltype(pc)::value;
+                k_up<R, PCv><<<grid, PCv * p->Q, smem, s>>>(src, uo, h, (const R*)p->m2m, p->P, p->Q);
+            });
+            LAUNCH_CHECK();
+            src = (const C*)outs(cur - h);
+            nbc >>= h;
+            cur -= h;
+        }
+        return FMMFFT_SUCCESS;
+    }
+
+    // ---- the whole far field per FMM p in one launch (G = 1): M2M, M2L-B, REDUCE, M2L + L2L
+    fmmfft_status_t tree_p() {
+        for (RankBufs& rb : p->ranks) {
+            TreePArgs a{};
+            for (int lev = p->B; lev <= p->L; ++lev) {
+                a.M[lev] = interior(rb.Mpad[lev]);
+                a.Lx[lev] = rb.Lloc[lev];
+                a.tab[lev] = p->m2l_pmaj[lev];
+            }
+            a.r = rb.r;
+            a.L = p->L;
+            a.B = p->B;
+            const int threads = sizeof(R) == 4 ? 1024 : 512;
+            const int maxo = (int)((((long long)p->Q << p->L) + threads - 1) / threads);
+            const size_t smem = tree_p_smem(p, threads);
+            dispatch<1, 2, 4, 8>(maxo <= 1 ? 1 : maxo <= 2 ? 2 : maxo <= 4 ? 4 : 8, [&](auto mo) {
+                constexpr int MO = decltype(mo)::value;
+                k_tree_p<R, MO><<<p->P - 1, threads, smem, s>>>(a, (const R*)p->m2m, p->P, p->Q,
+                                                                ((1 << p->B) - 3) * p->Q * p->Q);
+            });
+            LAUNCH_CHECK();
+        }
         return FMMFFT_SUCCESS;
     }
 
     // ---- m2m on own boxes, l = L-1 .. l_g
     fmmfft_status_t m2m_local() {
+        if (p->tree_p) return FMMFFT_SUCCESS;
         fmmfft_status_t st;
-        for (int lev = p->L - 1; lev >= p->lg; --lev)
-            for (RankBufs& rb : p->ranks)
-                if ((st = launch_m2m(interior(rb.Mpad[lev + 1]), interior(rb.Mpad[lev]), nb_at(lev)))) return st;
+        for (RankBufs& rb : p->ranks) {
+            auto outs = [&](int l) -> void* { return interior(rb.Mpad[l]); };
+            if ((st = launch_up(interior(rb.Mpad[p->L]), p->L, p->lg, nb_at(p->L), outs))) return st;
+        }
         return FMMFFT_SUCCESS;
     }
 
@@ -409,66 +563,131 @@ struct Exec {
         return FMMFFT_SUCCESS;
     }
 
+    // M2L + L2L for one interaction-list level (l > B)
     fmmfft_status_t launch_down(const C* src, long long src_base, int src_mod, const C* parent, long long par_base,
                                 C* outp, long long tgt_base, int ntg, int lev) {
-        const bool base = lev == p->B;
-        const int nshift = base ? (1 << p->B) - 3 : 3;
-        const R* tab = (const R*)(base ? p->m2lB : p->m2l[lev]);
+        const int PC_ = p->PCd;
+        const int npc = p->P / PC_;
+        // the table slice (4 Q^2 PC) is loaded once per CTA: prefer 16 targets per CTA, fewer
+        // only while that leaves most SMs idle
+        int BR = std::min(16, ntg);
+        while (BR > 4 && (long long)((ntg + BR - 1) / BR) * npc < 148) BR /= 2;
+        const size_t smem = (size_t)(BR + 4 + BR / 2) * p->Q * PC_ * sizeof(C) + (size_t)p->m2l_chunk * sizeof(R) +
+                            (size_t)2 * p->Q * p->Q * sizeof(R);
+        const dim3 grid((unsigned)((ntg + BR - 1) / BR), (unsigned)npc);
+        const R* tab = (const R*)p->m2l[lev];
+        with_pcd([&](auto pc) {
+            constexpr int PCv = decltype(pc)::value;
+            dispatch<2, 4, 8, 16>(BR, [&](auto br) {
+                constexpr int BRv = decltype(br)::value;
+                k_down<R, BRv, PCv><<<grid, PCv * p->Q, smem, s>>>(src, src_base, src_mod, parent, par_base, outp, tgt_base,
+                                                                   ntg, tab, p->m2l_chunk, (const R*)p->m2m, p->P, p->Q);
+            });
+        });
+        LAUNCH_CHECK();
+        return FMMFFT_SUCCESS;
+    }
+
+    // M2L-B + REDUCE on the gathered base level (sources: all 2^B boxes, periodic)
+    fmmfft_status_t launch_base(RankBufs& rb, C* outp, long long tgt_base, int ntg) {
+        const int nbB = 1 << p->B;
+        const int PC_ = p->PCd;
+        const size_t smem = ((size_t)nbB + 1) * p->Q * PC_ * sizeof(C) + (size_t)p->Q * p->Q * PC_ * sizeof(R);
+        if (ntg <= 32 && smem <= 200 * 1024) {
+            const int NTr = ntg <= 4 ? 4 : ntg <= 8 ? 8 : ntg <= 16 ? 16 : 32;
+            with_pcd([&](auto pc) {
+                constexpr int PCv = decltype(pc)::value;
+                dispatch<4, 8, 16, 32>(NTr, [&](auto ntv) {
+                    constexpr int NTv = decltype(ntv)::value;
+                    k_base<R, NTv, PCv><<<p->P / PCv, PCv * p->Q, smem, s>>>((const C*)rb.Mfull[p->B], outp, (C*)rb.r,
+                                                                           (int)tgt_base, ntg, (const R*)p->m2lB,
+                                                                           p->m2lB_chunk, nbB, p->P, p->Q);
+                });
+            });
+            LAUNCH_CHECK();
+            return FMMFFT_SUCCESS;
+        }
         const long long total = (long long)ntg * QP();
-        const int threads = 256;
-        const int blocks = (int)std::min<long long>((total + threads - 1) / threads, 148LL * 16);
-        const size_t smem = (size_t)2 * p->Q * p->Q * sizeof(R);
-        k_down<R><<<blocks, threads, smem, s>>>(src, src_base, src_mod, parent, par_base, outp, tgt_base, ntg, tab, nshift,
-                                                base ? 1 : 0, 1 << p->B, (const R*)p->m2m, p->P, p->Q);
+        const int blocks = (int)std::min<long long>((total + 255) / 256, 148LL * 16);
+        k_base_generic<R><<<blocks, 256, 0, s>>>((const C*)rb.Mfull[p->B], outp, tgt_base, ntg, (const R*)p->m2lB,
+                                                  p->m2lB_chunk, PC_, nbB, p->P, p->Q);
+        LAUNCH_CHECK();
+        k_reduce<R><<<(p->P + 127) / 128, 128, 0, s>>>((C*)rb.Mfull[p->B], (C*)rb.r, p->P, p->Q, nbB);
         LAUNCH_CHECK();
         return FMMFFT_SUCCESS;
     }
 
     // ---- top: replicated levels l_g .. B
     fmmfft_status_t top() {
+        if (p->tree_p) return tree_p();
         fmmfft_status_t st;
         for (RankBufs& rb : p->ranks) {
-            const int g = p->virt ? rb.g : g_comm.rank * (p->G > 1);
-            for (int lev = p->lg - 1; lev >= p->B; --lev)
-                if ((st = launch_m2m((C*)rb.Mfull[lev + 1], (C*)rb.Mfull[lev], 1 << lev))) return st;
-            // M2L-B: targets = own boxes if l_g == B, else all 2^B boxes
-            if (p->lg == p->B) {
-                if ((st = launch_down((C*)rb.Mfull[p->B], 0, 1 << p->B, nullptr, 0, (C*)rb.Lloc[p->B],
-                                      (long long)g * nb_at(p->B), nb_at(p->B), p->B))) return st;
-            } else {
-                if ((st = launch_down((C*)rb.Mfull[p->B], 0, 1 << p->B, nullptr, 0, (C*)rb.Lfull[p->B], 0, 1 << p->B, p->B)))
-                    return st;
+            const int g = grank(rb);
+            if (p->lg > p->B) {
+                auto outs = [&](int l) -> void* { return rb.Mfull[l]; };
+                if ((st = launch_up((C*)rb.Mfull[p->lg], p->lg, p->B, 1LL << p->lg, outs))) return st;
             }
-            k_reduce<R><<<(p->P + 127) / 128, 128, 0, s>>>((C*)rb.Mfull[p->B], (C*)rb.r, p->P, p->Q, 1 << p->B);
-            LAUNCH_CHECK();
-            for (int lev = p->B + 1; lev <= p->lg; ++lev) {
-                if (lev < p->lg) {
-                    if ((st = launch_down((C*)rb.Mfull[lev], 0, 1 << lev, (C*)rb.Lfull[lev - 1], 0, (C*)rb.Lfull[lev], 0,
-                                          1 << lev, lev))) return st;
-                } else {
-                    if ((st = launch_down((C*)rb.Mfull[lev], 0, 1 << lev, (C*)rb.Lfull[lev - 1], 0, (C*)rb.Lloc[lev],
-                                          (long long)g * nb_at(lev), nb_at(lev), lev))) return st;
-                }
+            // M2L-B (+ REDUCE): targets = own boxes if l_g == B, else all 2^B boxes
+            if (p->lg == p->B) {
+                if ((st = launch_base(rb, (C*)rb.Lloc[p->B], (long long)g * nb_at(p->B), nb_at(p->B)))) return st;
+            } else {
+                if ((st = launch_base(rb, (C*)rb.Lfull[p->B], 0, 1 << p->B))) return st;
             }
         }
         return FMMFFT_SUCCESS;
     }
 
-    // ---- down: distributed levels l_g+1 .. L
+    // ---- down: M2L + L2L for every level B+1 .. L in one launch per rank (k_tree_down)
     fmmfft_status_t down() {
-        fmmfft_status_t st;
-        for (int lev = p->lg + 1; lev <= p->L; ++lev) {
-            for (RankBufs& rb : p->ranks) {
-                const int g = p->virt ? rb.g : g_comm.rank * (p->G > 1);
-                const long long nbl = nb_at(lev), nbp = nb_at(lev - 1);
-                const C* src;
-                long long src_base;
-                int mod;
-                if (p->G == 1) { src = interior(rb.Mpad[lev]); src_base = 0; mod = 1 << lev; }
-                else { src = (C*)rb.Mpad[lev]; src_base = g * nbl - 2; mod = 0; }
-                if ((st = launch_down(src, src_base, mod, (C*)rb.Lloc[lev - 1], g * nbp, (C*)rb.Lloc[lev], g * nbl, (int)nbl,
-                                      lev))) return st;
+        if (p->L == p->B || p->tree_p) return FMMFFT_SUCCESS;
+        const int PC_ = p->PCd;
+        const int npc = p->P / PC_;
+        const int QPC = p->Q * PC_;
+        int optin = 0;
+        CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, p->device));
+        auto smem_of = [&](int nr, int db) {
+            return (size_t)(1 + db) * p->m2l_chunk * sizeof(R) + (size_t)(1 + db) * (nr + 6) * QPC * sizeof(C) +
+                   (size_t)nr * QPC * sizeof(C) + (size_t)(nr / 2 + 1) * QPC * sizeof(C) + (size_t)2 * p->Q * p->Q * sizeof(R);
+        };
+        int NR = std::min(16, p->nb);
+        while (NR > 1 && (long long)(p->nb / NR) * npc < 148) NR /= 2;
+        while (NR > 1 && smem_of(NR, 0) > (size_t)optin) NR /= 2;
+        const int db = smem_of(NR, 1) <= (size_t)optin ? 1 : 0;
+        const size_t smem = smem_of(NR, db);
+        for (RankBufs& rb : p->ranks) {
+            const long long g = grank(rb);
+            TreeDownArgs a{};
+            for (int lev = p->B + 1; lev <= p->L; ++lev) {
+                TreeLevel& tl = a.lev[lev];
+                const long long nbl = nb_at(lev);
+                tl.tab = p->m2l[lev];
+                if (p->G == 1) {
+                    tl.src = interior(rb.Mpad[lev]); tl.src_base = 0; tl.src_mod = 1 << lev;
+                    tl.out = rb.Lloc[lev]; tl.out_base = 0;
+                } else if (lev <= p->lg) {
+                    tl.src = rb.Mfull[lev]; tl.src_base = 0; tl.src_mod = 1 << lev;
+                    if (lev == p->lg) { tl.out = rb.Lloc[lev]; tl.out_base = g * nbl; }
+                    else { tl.out = rb.Lfull[lev]; tl.out_base = 0; }
+                } else {
+                    tl.src = rb.Mpad[lev]; tl.src_base = g * nbl - 2; tl.src_mod = 0;
+                    tl.out = rb.Lloc[lev]; tl.out_base = g * nbl;
+                }
             }
+            if (p->lg == p->B) { a.par0 = rb.Lloc[p->B]; a.par0_base = g * nb_at(p->B); }
+            else { a.par0 = rb.Lfull[p->B]; a.par0_base = 0; }
+            a.leaf0 = g * p->nb;
+            a.lstart = p->B + 1;
+            a.L = p->L;
+            const dim3 grid((unsigned)(p->nb / NR), (unsigned)npc);
+            with_pcd([&](auto pc) {
+                constexpr int PCv = decltype(pc)::value;
+                dispatch<1, 2, 4, 8, 16>(NR, [&](auto nr) {
+                    constexpr int NRv = decltype(nr)::value;
+                    k_tree_down<R, PCv, NRv><<<grid, PCv * p->Q, smem, s>>>(a, (const R*)p->m2m, p->P, p->Q,
+                                                                            p->m2l_chunk, db);
+                });
+            });
+            LAUNCH_CHECK();
         }
         return FMMFFT_SUCCESS;
     }
@@ -476,13 +695,16 @@ struct Exec {
     // ---- L2T + POST + P-FFT
     fmmfft_status_t post_pfft() {
         const int MS = std::min(p->M_L, std::max(1, TILE / p->P));
+        const int threads = std::min(sizeof(R) == 4 ? 1024 : 512, std::max(32, MS * p->P / 8));
         const size_t smem = (size_t)MS * (p->P + 1) * sizeof(C) + (size_t)p->P * sizeof(C) + (size_t)p->Q * MS * sizeof(R);
-        CUDA_TRY(cudaFuncSetAttribute(k_post_pfft<R, EPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         const int blocks = p->nb * (p->M_L / MS);
         for (RankBufs& rb : p->ranks) {
-            k_post_pfft<R, EPT><<<blocks, 256, smem, s>>>((const C*)rb.Tn, (const C*)rb.Lloc[p->L], (const C*)rb.r,
-                                                         (const C*)p->rho, (const R*)p->s2m, (C*)rb.W, p->P, p->M_L, p->Q, MS,
-                                                         p->Mg);
+            dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 11>(ilog2(p->P), [&](auto lp) {
+                constexpr int LP = decltype(lp)::value;
+                k_post_pfft<R, LP><<<blocks, threads, smem, s>>>((const C*)rb.Tn, (const C*)rb.Lloc[p->L], (const C*)rb.r,
+                                                                (const C*)p->rho, (const R*)p->s2m, (C*)rb.W,
+                                                                ilog2(p->M_L), p->Q, ilog2(MS), (int)p->Mg);
+            });
             LAUNCH_CHECK();
         }
         return FMMFFT_SUCCESS;
@@ -515,28 +737,32 @@ struct Exec {
     fmmfft_status_t mfft() {
         const int n = (int)p->radices.size();
         const long long rows = p->P / p->G;
+        const int lM = ilog2(p->M);
         for (RankBufs& rb : p->ranks) {
             C* dst = out[p->virt ? rb.g : 0];
             const C* src = (const C*)(p->G > 1 ? rb.Rcv : rb.W);
-            long long Ns = 1;
+            int lNs = 0;
             for (int i = 0; i < n; ++i) {
-                const int Rp = p->radices[i];
+                const int Rp = p->radices[i], lR = ilog2(Rp);
                 C* o = ((n - 1 - i) % 2 == 0) ? dst : (C*)rb.tmp;
                 const long long nj = p->M / Rp;
-                int c = (int)std::min<long long>(TILE / Rp, nj);
-                while (c > 8 && (nj / c) * rows < 2 * 148) c /= 2;
-                long long in_row = p->M, blk = p->M, blk_stride = 0;
+                long long c = std::min<long long>(TILE / Rp, nj);
+                while (c > 8 && c * Rp > 2048 && (nj / c) * rows < 2 * 148) c /= 2;
+                int in_row = (int)p->M, lblk = lM, blk_stride = 0;
                 if (i == 0 && p->G > 1) {
-                    in_row = p->Mg; blk = p->Mg; blk_stride = (long long)(p->P / p->G) * p->Mg;
-                    c = (int)std::min<long long>(c, p->Mg);
+                    in_row = (int)p->Mg; lblk = ilog2(p->Mg); blk_stride = (int)((p->P / p->G) * p->Mg);
+                    c = std::min<long long>(c, p->Mg);
                 }
+                const int threads = (int)std::min<long long>(sizeof(R) == 4 ? 1024 : 512, std::max<long long>(32, c * Rp / 8));
                 const size_t smem = (size_t)c * (Rp + 1) * sizeof(C) + (size_t)Rp * sizeof(C);
-                CUDA_TRY(cudaFuncSetAttribute(k_fft_pass<R, EPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
                 const dim3 grid((unsigned)(nj / c), (unsigned)rows);
-                k_fft_pass<R, EPT><<<grid, 256, smem, s>>>(src, o, p->M, Rp, Ns, c, in_row, blk, blk_stride);
+                dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10>(lR, [&](auto lr) {
+                    constexpr int LR = decltype(lr)::value;
+                    k_fft_pass<R, LR><<<grid, threads, smem, s>>>(src, o, lM, lNs, ilog2(c), in_row, lblk, blk_stride);
+                });
                 LAUNCH_CHECK();
                 src = o;
-                Ns *= Rp;
+                lNs += lR;
             }
         }
         return FMMFFT_SUCCESS;
@@ -561,21 +787,61 @@ struct Exec {
 
 template <typename R>
 static fmmfft_status_t execute_t(fmmfft_plan_s* p, const void* in, void* out, cudaStream_t s) {
-    Exec<R> ex{p, s, {}, {}};
-    const long long nl = p->N / p->G;
-    if (p->virt) {
-        for (int g = 0; g < p->G; ++g) {
-            ex.in.push_back((const C2<R>*)in + g * nl);
-            ex.out.push_back((C2<R>*)out + g * nl);
-        }
-    } else {
-        ex.in.push_back((const C2<R>*)in);
-        ex.out.push_back((C2<R>*)out);
+    // replay a captured graph for this (in, out) pair
+    if (p->use_graph) {
+        for (auto& ge : p->graphs)
+            if (ge.in == in && ge.out == out) {
+                CUDA_TRY(cudaGraphLaunch(ge.exec, s));
+                p->kernels = ge.nlaunch;
+                p->have_times = (p->flags & FMMFFT_FLAG_PROFILE) != 0;
+                return FMMFFT_SUCCESS;
+            }
     }
+    const long long nl = p->N / p->G;
+    auto make = [&](cudaStream_t st) {
+        Exec<R> ex{p, st, {}, {}};
+        if (p->virt) {
+            for (int g = 0; g < p->G; ++g) {
+                ex.in.push_back((const C2<R>*)in + g * nl);
+                ex.out.push_back((C2<R>*)out + g * nl);
+            }
+        } else {
+            ex.in.push_back((const C2<R>*)in);
+            ex.out.push_back((C2<R>*)out);
+        }
+        return ex;
+    };
+    if (!p->use_graph) {
+        Exec<R> ex = make(s);
+        fmmfft_status_t st = ex.run();
+        p->kernels = ex.nlaunch;
+        p->have_times = st == FMMFFT_SUCCESS && (p->flags & FMMFFT_FLAG_PROFILE);
+        return st;
+    }
+    // capture on the plan's own stream (the caller's may be the legacy default stream)
+    Exec<R> ex = make(p->cap_stream);
+    CUDA_TRY(cudaStreamBeginCapture(p->cap_stream, cudaStreamCaptureModeRelaxed));
     fmmfft_status_t st = ex.run();
-    p->last_stream = s;
-    p->have_times = st == FMMFFT_SUCCESS && (p->flags & FMMFFT_FLAG_PROFILE);
-    return st;
+    cudaGraph_t graph = nullptr;
+    cudaError_t e = cudaStreamEndCapture(p->cap_stream, &graph);
+    if (st) {
+        if (graph) cudaGraphDestroy(graph);
+        return st;
+    }
+    CUDA_TRY(e);
+    cudaGraphExec_t exec = nullptr;
+    e = cudaGraphInstantiate(&exec, graph, 0);
+    cudaGraphDestroy(graph);
+    CUDA_TRY(e);
+    if (p->graphs.size() >= 8) {
+        cudaGraphExecDestroy(p->graphs.front().exec);
+        p->graphs.erase(p->graphs.begin());
+    }
+    p->graphs.push_back(GraphEntry{in, out, exec, ex.nlaunch});
+    CUDA_TRY(cudaGraphLaunch(exec, s));
+    p->kernels = ex.nlaunch;
+    p->have_times = (p->flags & FMMFFT_FLAG_PROFILE) != 0;
+    return FMMFFT_SUCCESS;
 }
 
 }  // namespace fmmfft
@@ -586,7 +852,7 @@ using namespace fmmfft;
 extern "C" {
 
 const char* fmmfft_last_error(void) { return g_last_error.c_str(); }
-const char* fmmfft_version(void) { return "fmmfft-b200 0.1 (sm_100a)"; }
+const char* fmmfft_version(void) { return "fmmfft-b200 0.2 (sm_100a)"; }
 const char* fmmfft_stage_name(int i) { return (i >= 0 && i < ST_COUNT) ? kStageNames[i] : ""; }
 
 fmmfft_status_t fmmfft_get_unique_id(unsigned char id[128]) {
@@ -635,6 +901,7 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
     if (M_L < 16 || M_L > 128) return fail(FMMFFT_INVALID_VALUE, "need 16 <= M_L <= 128");
     if (Q < 2 || Q > 32) return fail(FMMFFT_INVALID_VALUE, "need 2 <= Q <= 32");
     if (N % ((long long)P * M_L)) return fail(FMMFFT_INVALID_VALUE, "N must be a multiple of P*M_L");
+    if (N / G > (1LL << 30)) return fail(FMMFFT_UNSUPPORTED, "N/G > 2^30 per rank not supported");
     const long long nleaf = N / ((long long)P * M_L);
     const int L = ilog2(nleaf);
     if (B < 2 || L < B) return fail(FMMFFT_INVALID_VALUE, "need L >= B >= 2 (L=%d, B=%d)", L, B);
@@ -651,6 +918,8 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
     CUDA_TRY(cudaGetDeviceProperties(&prop, dev));
     if (prop.major != 10 || prop.minor != 0)
         return fail(FMMFFT_UNSUPPORTED, "device %s is sm_%d%d; this build is sm_100a only", prop.name, prop.major, prop.minor);
+    fmmfft_status_t st = precision == FMMFFT_C64 ? init_kernel_attrs<float>() : init_kernel_attrs<double>();
+    if (st) return st;
 
     fmmfft_plan_s* p = new fmmfft_plan_s;
     p->N = N; p->P = P; p->G = G; p->B = B; p->Q = Q; p->M_L = M_L; p->L = L;
@@ -660,8 +929,21 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
     if (G == 1) p->lg = B;
     p->esz = precision == FMMFFT_C64 ? 8 : 16;
     p->rsz = p->esz / 2;
+    p->PCn = std::min(P, precision == FMMFFT_C64 ? 32 : 16);
+    p->PCd = std::min(P, precision == FMMFFT_C64 ? 16 : 8);
+    // fused per-FMM far field (k_tree_p) for single-GPU plans whose tree fits one CTA's
+    // shared memory and at most 8 outputs per thread per level
+    {
+        const int threads = precision == FMMFFT_C64 ? 1024 : 512;
+        int optin = 0;
+        cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+        p->tree_p = (G == 1) && ((long long)Q << L) <= 8LL * threads && tree_p_smem(p, threads) <= (size_t)optin;
+        if (const char* e = getenv("FMMFFT_TREE")) p->tree_p = p->tree_p && e[0] == 'p';
+    }
+    const char* g_env = getenv("FMMFFT_NO_GRAPH");
+    p->use_graph = !(g_env && g_env[0] == '1');
     plan_radices(p);
-    fmmfft_status_t st = precision == FMMFFT_C64 ? build_tables<float>(p) : build_tables<double>(p);
+    st = precision == FMMFFT_C64 ? build_tables<float>(p) : build_tables<double>(p);
     if (!st) {
         const int nr = virt ? G : 1;
         p->ranks.resize(nr);
@@ -677,11 +959,14 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
         }
     }
     if (!st) {
+        cudaError_t e = cudaStreamCreateWithFlags(&p->cap_stream, cudaStreamNonBlocking);
+        if (e != cudaSuccess) st = fail(FMMFFT_CUDA_ERROR, "cudaStreamCreate: %s", cudaGetErrorString(e));
+    }
+    if (!st) {
         cudaError_t e = cudaDeviceSynchronize();
         if (e != cudaSuccess) st = fail(FMMFFT_CUDA_ERROR, "plan setup: %s", cudaGetErrorString(e));
     }
     if (st) { destroy_plan(p); return st; }
-    p->kernels = count_kernels(p);
     *plan = p;
     return FMMFFT_SUCCESS;
 }

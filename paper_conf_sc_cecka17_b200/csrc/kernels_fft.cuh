@@ -5,7 +5,9 @@
 //     L2T -> POST -> FFT_P -> transposed store is one kernel);
 //   * k_fft_pass: one pass of a multi-pass Stockham FFT over rows of length M (§3 step 4),
 //     the first pass reading the all-to-all receive layout directly.
-// Both use the same shared-memory Stockham autosort FFT on a tile of `ncols` columns.
+// Both run the same shared-memory Stockham autosort FFT on a tile of columns, compiled for one
+// transform length (template LLEN = log2 length): every stage's radix, shifts, masks and
+// twiddle strides are compile-time constants; 8 elements per thread per stage.
 #pragma once
 #include "common.cuh"
 
@@ -43,30 +45,53 @@ template <int E, typename C> __device__ __forceinline__ void dftE(C* v) {
     else dft8(v);
 }
 
-// One radix-E Stockham stage on a shared tile: columns col < ncols of length len (power of
-// two), column stride ld. For each butterfly j < len/E with k = j mod Ns:
+// exp(-2 pi i e / 2^ls) for 0 <= e < 2^ls, exact argument (split above 2^24 for fp32)
+__device__ __forceinline__ float2 twiddle_pow2(float, int e, int ls) {
+    float s, c;
+    if (ls <= 24) {
+        sincospif(ldexpf((float)e, 1 - ls), &s, &c);
+        return make_float2(c, -s);
+    }
+    const int hi = e & ~4095, lo = e & 4095;
+    float s2, c2;
+    sincospif(ldexpf((float)hi, 1 - ls), &s, &c);
+    sincospif(ldexpf((float)lo, 1 - ls), &s2, &c2);
+    return cmul(make_float2(c, -s), make_float2(c2, -s2));
+}
+__device__ __forceinline__ double2 twiddle_pow2(double, int e, int ls) {
+    double s, c;
+    sincospi(ldexp((double)e, 1 - ls), &s, &c);
+    return make_double2(c, -s);
+}
+
+// One radix-E Stockham stage on a shared tile of columns of length 2^LLEN, column stride
+// 2^LLEN + 1 (padding against bank conflicts). For each butterfly j < len/E, k = j mod Ns:
 //   v_t = x[j + t len/E] w_{Ns E}^{k t};  v = DFT_E(v);  y[(j - k) E + k + t Ns] = v_t.
-// In place: each thread keeps its butterflies' values in registers across a barrier.
-// tw[u] = w_len^u for u < len. EPT = elements per thread (ncols * len <= EPT * blockDim).
-template <int E, int EPT, typename C>
-__device__ __forceinline__ void stockham_stage(C* tile, int ncols, int len, int ld, int Ns, const C* tw) {
-    constexpr int NB = EPT / E;
+// In place: each thread keeps its 8/E butterflies in registers across a barrier.
+// tw[u] = w_len^u, u < len.
+template <int E, int LLEN, int LNS, typename C>
+__device__ __forceinline__ void stockham_stage(C* tile, int ncols, const C* tw) {
+    constexpr int NB = 8 / E;
+    constexpr int LE = E == 8 ? 3 : (E == 4 ? 2 : 1);
+    constexpr int LPER = LLEN - LE;
+    constexpr int LD = (1 << LLEN) + 1;
+    constexpr int NS = 1 << LNS;
+    constexpr int LTWS = LLEN - LNS - LE;                       // tw index = k t len / (Ns E)
     const int nthr = blockDim.x, tid = threadIdx.x;
-    const int per = len / E;
-    const int total = ncols * per;
-    const int tws = len / (Ns * E);
+    const int total = ncols << LPER;
     C v[NB][E];
 #pragma unroll
     for (int k = 0; k < NB; ++k) {
         const int bf = tid + k * nthr;
         if (bf < total) {
-            const int col = bf / per, j = bf % per, kk = j % Ns;
-            const C* x = tile + col * ld + j;
+            const int col = bf >> LPER, j = bf & ((1 << LPER) - 1);
+            const C* x = tile + col * LD + j;
 #pragma unroll
-            for (int t = 0; t < E; ++t) v[k][t] = x[t * per];
-            if (Ns > 1) {
+            for (int t = 0; t < E; ++t) v[k][t] = x[t << LPER];
+            if constexpr (LNS > 0) {
+                const int kk = j & (NS - 1);
 #pragma unroll
-                for (int t = 1; t < E; ++t) v[k][t] = cmul(v[k][t], tw[(kk * t * tws) & (len - 1)]);
+                for (int t = 1; t < E; ++t) v[k][t] = cmul(v[k][t], tw[(kk * t) << LTWS]);
             }
             dftE<E>(v[k]);
         }
@@ -76,30 +101,29 @@ __device__ __forceinline__ void stockham_stage(C* tile, int ncols, int len, int 
     for (int k = 0; k < NB; ++k) {
         const int bf = tid + k * nthr;
         if (bf < total) {
-            const int col = bf / per, j = bf % per, kk = j % Ns;
-            C* y = tile + col * ld + (j - kk) * E + kk;
+            const int col = bf >> LPER, j = bf & ((1 << LPER) - 1), kk = j & (NS - 1);
+            C* y = tile + col * LD + ((j - kk) << LE) + kk;
 #pragma unroll
-            for (int t = 0; t < E; ++t) y[t * Ns] = v[k][t];
+            for (int t = 0; t < E; ++t) y[t << LNS] = v[k][t];
         }
     }
     __syncthreads();
 }
 
-// Full in-place FFT of every column: radix-8 stages, then one radix-4 or radix-2 stage.
-template <int EPT, typename C>
-__device__ void fft_columns(C* tile, int ncols, int len, int ld, const C* tw) {
-    int Ns = 1;
-    while (Ns < len) {
-        const int rem = len / Ns;
-        if (rem >= 8) { stockham_stage<8, EPT>(tile, ncols, len, ld, Ns, tw); Ns *= 8; }
-        else if (rem == 4) { stockham_stage<4, EPT>(tile, ncols, len, ld, Ns, tw); Ns *= 4; }
-        else { stockham_stage<2, EPT>(tile, ncols, len, ld, Ns, tw); Ns *= 2; }
+// In-place FFT of every column: radix-8 stages, then one radix-4 or radix-2 stage.
+template <int LLEN, int LNS = 0, typename C>
+__device__ __forceinline__ void fft_columns(C* tile, int ncols, const C* tw) {
+    if constexpr (LNS < LLEN) {
+        constexpr int REM = LLEN - LNS;
+        constexpr int LE = REM >= 3 ? 3 : REM;
+        stockham_stage<1 << LE, LLEN, LNS>(tile, ncols, tw);
+        fft_columns<LLEN, LNS + LE>(tile, ncols, tw);
     }
 }
 
 template <typename R>
-__device__ __forceinline__ void fill_twiddles(C2<R>* tw, int len) {
-    for (int u = threadIdx.x; u < len; u += blockDim.x) tw[u] = twiddle<R>(u, len);
+__device__ __forceinline__ void fill_twiddles(C2<R>* tw, int llen) {
+    for (int u = threadIdx.x; u < (1 << llen); u += blockDim.x) tw[u] = twiddle_pow2(R(0), u, llen);
 }
 
 // ---------------------------------------------------------------------------------------------
@@ -107,29 +131,31 @@ __device__ __forceinline__ void fill_twiddles(C2<R>* tw, int len) {
 //   T_{pmb}  = T_near_{pmb} + L2T_{mq} L^L_{pqb}                       p >= 1
 //   T_{pmb} <- rho_p (T_{pmb} + i r_p)                                   p >= 1   (R1)
 //   W[k2][m] = sum_p w_P^{p k2} T_{pm}
-// CTA = (leaf box b, m sub-tile of MS rows). W row k2 has length M/G (this rank's m range):
-// element (k2, m_local) at W[k2 * Mg + m_local] — which is the all-to-all send layout
-// [destination r][k2 local][m local] with k2 = r P/G + k2 local.
+// CTA = (leaf box b, m sub-tile of MS rows), MS*P/8 threads, P = 2^LP. W row k2 has length
+// Mg = M/G (this rank's m range): element (k2, m_local) at W[k2 * Mg + m_local] — the
+// all-to-all send layout [destination r][k2 local][m local] with k2 = r P/G + k2 local.
 // ---------------------------------------------------------------------------------------------
-template <typename R, int EPT>
-__global__ void __launch_bounds__(256)
+template <typename R, int LP>
+__global__ void __launch_bounds__(sizeof(R) == 4 ? 1024 : 512)
 k_post_pfft(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2<R>* __restrict__ r,
             const C2<R>* __restrict__ rho, const R* __restrict__ s2m, C2<R>* __restrict__ W,
-            int P, int M_L, int Q, int MS, long long Mg) {
+            int lML, int Q, int lMS, int Mg) {
     using C = C2<R>;
+    constexpr int P = 1 << LP, LD = P + 1;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    const int ld = P + 1;
+    const int MS = 1 << lMS, M_L = 1 << lML;
     C* tile = reinterpret_cast<C*>(smem_raw);                    // [MS][P + 1]
-    C* tw = tile + MS * ld;                                       // [P]
+    C* tw = tile + MS * LD;                                       // [P]
     R* s2m_sm = reinterpret_cast<R*>(tw + P);                    // [Q][MS]
     const int tid = threadIdx.x, nthr = blockDim.x;
-    const int nsub = M_L / MS;
-    const int b = blockIdx.x / nsub, m0 = (blockIdx.x % nsub) * MS;
+    const int lnsub = lML - lMS;
+    const int b = blockIdx.x >> lnsub, m0 = (blockIdx.x & ((1 << lnsub) - 1)) << lMS;
 
-    fill_twiddles<R>(tw, P);
-    for (int idx = tid; idx < Q * MS; idx += nthr) s2m_sm[idx] = s2m[(idx / MS) * M_L + m0 + idx % MS];
-    const C* src = Tn + ((size_t)b * M_L + m0) * P;
-    for (int idx = tid; idx < MS * P; idx += nthr) tile[(idx / P) * ld + idx % P] = ldg_c(src + idx);
+    const C* src = Tn + (((size_t)b << lML) + m0) * P;
+    for (int idx = tid; idx < (MS << LP); idx += nthr) cp_async_elem(tile + (idx >> LP) * LD + (idx & (P - 1)), src + idx);
+    for (int idx = tid; idx < Q * MS; idx += nthr) cp_async_elem(s2m_sm + idx, s2m + (idx >> lMS) * M_L + m0 + (idx & (MS - 1)));
+    fill_twiddles<R>(tw, LP);
+    cp_async_wait_all();
     __syncthreads();
 
     // L2T + POST: thread owns one p and a group of MG consecutive m (L^L loaded once per q).
@@ -137,13 +163,13 @@ k_post_pfft(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2
     const int ngrp = (MS + MG - 1) / MG;
     const C* Lb = LL + (size_t)b * Q * P;
     for (int idx = tid; idx < P * ngrp; idx += nthr) {
-        const int p = idx % P, g = idx / P;
+        const int p = idx & (P - 1), g = idx >> LP;
         if (p == 0) continue;                                      // C_0 = I (R1)
         C acc[MG];
 #pragma unroll
         for (int u = 0; u < MG; ++u) acc[u] = zero<C>();
         for (int q = 0; q < Q; ++q) {
-            const C l = ldg_c(Lb + (size_t)q * P + p);
+            const C l = ldg_c(Lb + q * P + p);
 #pragma unroll
             for (int u = 0; u < MG; ++u)
                 if (g * MG + u < MS) rfma(acc[u], s2m_sm[q * MS + g * MG + u], l);
@@ -153,74 +179,91 @@ k_post_pfft(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2
         for (int u = 0; u < MG; ++u) {
             const int m = g * MG + u;
             if (m < MS) {
-                C t = cadd(tile[m * ld + p], acc[u]);
+                C t = cadd(tile[m * LD + p], acc[u]);
                 t.x -= rp.y; t.y += rp.x;                           // + i r_p
-                tile[m * ld + p] = cmul(rh, t);
+                tile[m * LD + p] = cmul(rh, t);
             }
         }
     }
     __syncthreads();
-    fft_columns<EPT>(tile, MS, P, ld, tw);
+    fft_columns<LP>(tile, MS, tw);
     // W[k2][b M_L + m0 + m]: contiguous runs of MS along m for every k2
-    C* dst = W + (size_t)b * M_L + m0;
-    for (int idx = tid; idx < MS * P; idx += nthr) {
-        const int k2 = idx / MS, m = idx % MS;
-        dst[(size_t)k2 * Mg + m] = tile[m * ld + k2];
+    C* dst = W + ((size_t)b << lML) + m0;
+    for (int idx = tid; idx < (MS << LP); idx += nthr) {
+        const int k2 = idx >> lMS, m = idx & (MS - 1);
+        dst[(size_t)k2 * Mg + m] = tile[m * LD + k2];
     }
 }
 
 // ---------------------------------------------------------------------------------------------
-// One pass of the multi-pass Stockham FFT along rows of length M (§3 step 4):
-// radix Rp, span Ns (product of the previous passes' radices). For j < M/Rp, k = j mod Ns:
+// One pass of the multi-pass Stockham FFT along rows of length M = 2^lM (§3 step 4):
+// radix Rp = 2^LR, span Ns = 2^lNs (product of the previous passes' radices). For j < M/Rp,
+// k = j mod Ns:
 //   v_t = x[j + t M/Rp] w_{Ns Rp}^{k t},  v = DFT_Rp(v),  y[(j - k) Rp + k + t Ns] = v_t.
-// CTA = (chunk of c consecutive j, row). Element m of input row `row` is read at
-//   in[row * in_row + (m / blk) * blk_stride + m % blk]
-// which expresses both a plain row (blk = M) and the all-to-all receive layout
-// [source rank][k2 local][m local] (blk = M/G, blk_stride = (P/G)(M/G), in_row = M/G).
-// Output rows are plain: out[row * M + index].
+// CTA = (chunk of c = 2^lc consecutive j, row), c*Rp/8 threads. Input element m of row `row`
+// is at in[row * in_row + (m >> lblk) * blk_stride + (m & (2^lblk - 1))], which expresses both a
+// plain row (lblk = lM) and the all-to-all receive layout [source rank][k2 local][m local]
+// (2^lblk = M/G, blk_stride = (P/G)(M/G), in_row = M/G). Output rows are plain.
 // ---------------------------------------------------------------------------------------------
-template <typename R, int EPT>
-__global__ void __launch_bounds__(256)
-k_fft_pass(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, long long M, int Rp, long long Ns, int c,
-           long long in_row, long long blk, long long blk_stride) {
+template <typename R, int LR>
+__global__ void __launch_bounds__(sizeof(R) == 4 ? 1024 : 512)
+k_fft_pass(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, int lM, int lNs, int lc,
+           int in_row, int lblk, int blk_stride) {
     using C = C2<R>;
+    constexpr int Rp = 1 << LR, LD = Rp + 1;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    const int ld = Rp + 1;
+    const int c = 1 << lc;
     C* tile = reinterpret_cast<C*>(smem_raw);                    // [c][Rp + 1]
-    C* tw = tile + c * ld;                                        // [Rp]
+    C* tw = tile + c * LD;                                        // [Rp]
     const int tid = threadIdx.x, nthr = blockDim.x;
-    const long long row = blockIdx.y;
-    const long long j0 = (long long)blockIdx.x * c;
-    const long long stride = M / Rp;
-    const long long span = Ns * Rp;
+    const size_t row = blockIdx.y;
+    const int j0 = blockIdx.x << lc;
+    const int lstride = lM - LR;
+    const int Ns = 1 << lNs;
+    const int lspan = lNs + LR;
+    const int bmask = (1 << lblk) - 1;
+    const C* xin = in + row * (size_t)in_row;
+    const int total = c << LR;
 
-    fill_twiddles<R>(tw, Rp);
-    const C* xin = in + row * in_row;
-    for (int idx = tid; idx < c * Rp; idx += nthr) {
-        const int t = idx / c, jj = idx % c;
-        const long long m = j0 + jj + (long long)t * stride;
-        C v = ldg_c(xin + (m / blk) * blk_stride + (m % blk));
-        if (Ns > 1) {
-            const long long k = (j0 + jj) % Ns;
-            if (t) v = cmul(v, twiddle<R>((k * t) % span, span));
+    // 8 elements per thread: all loads issued before any is used
+    C v[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+        const int idx = tid + u * nthr;
+        if (idx < total) {
+            const int t = idx >> lc, jj = idx & (c - 1);
+            const int m = j0 + jj + (t << lstride);
+            v[u] = ldg_c(xin + (size_t)(m >> lblk) * blk_stride + (m & bmask));
         }
-        tile[jj * ld + t] = v;
+    }
+    fill_twiddles<R>(tw, LR);
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+        const int idx = tid + u * nthr;
+        if (idx < total) {
+            const int t = idx >> lc, jj = idx & (c - 1);
+            C x = v[u];
+            if (lNs > 0 && t) x = cmul(x, twiddle_pow2(R(0), ((j0 + jj) & (Ns - 1)) * t, lspan));
+            tile[jj * LD + t] = x;
+        }
     }
     __syncthreads();
-    fft_columns<EPT>(tile, c, Rp, ld, tw);
-    C* yout = out + row * M;
-    if (Ns >= c) {
-        for (int idx = tid; idx < c * Rp; idx += nthr) {
-            const int t = idx / c, jj = idx % c;
-            const long long j = j0 + jj, k = j % Ns;
-            yout[(j - k) * Rp + k + (long long)t * Ns] = tile[jj * ld + t];
+    fft_columns<LR>(tile, c, tw);
+    C* yout = out + (row << lM);
+    if (lNs >= lc) {
+#pragma unroll 4
+        for (int idx = tid; idx < total; idx += nthr) {
+            const int t = idx >> lc, jj = idx & (c - 1);
+            const int j = j0 + jj, k = j & (Ns - 1);
+            yout[((j - k) << LR) + k + (t << lNs)] = tile[jj * LD + t];
         }
     } else {
-        const int ns = (int)Ns;
-        for (int idx = tid; idx < c * Rp; idx += nthr) {
-            const int jb = idx / (ns * Rp), rem = idx % (ns * Rp);
-            const int t = rem / ns, k = rem % ns;
-            yout[j0 * Rp + idx] = tile[(jb * ns + k) * ld + t];
+        const int lblkw = lNs + LR;
+#pragma unroll 4
+        for (int idx = tid; idx < total; idx += nthr) {
+            const int jb = idx >> lblkw, rem = idx & ((1 << lblkw) - 1);
+            const int t = rem >> lNs, k = rem & (Ns - 1);
+            yout[(j0 << LR) + idx] = tile[((jb << lNs) + k) * LD + t];
         }
     }
 }

@@ -186,7 +186,7 @@ def test_profile_stage_times(F):
     t = plan.stage_times()
     assert list(t) == ["comm_S", "near_up", "m2m", "comm_M", "top", "down", "post_pfft", "a2a", "mfft"]
     assert all(v >= 0 for v in t.values()) and t["near_up"] > 0
-    assert plan.info["kernels_per_execute"] > 5
+    assert plan.info["kernels_per_execute"] >= 4
 
 
 # ------------------------------------------------------------------ full-size bench configs, sampled
