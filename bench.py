@@ -43,12 +43,11 @@ def flops_fft(N: int) -> float:
     return 5.0 * N * math.log2(N)
 
 
-def near_up_flops(N, P, B, Q, M_L, G, C=2):
-    """Algorithmic flops of one near_up launch (S2T + S2M, §5.1), per rank."""
+def s2t_flops(N, P, M_L, G, C=2):
+    """Algorithmic flops of one S2T launch (the near field, §5.1 P:1165-1167:
+    6 C M_L^2 2^L (P-1) / G), per rank."""
     L = int(round(math.log2(N // (P * M_L))))
-    s2t = 6 * C * M_L * M_L * 2 ** L * (P - 1) / G
-    s2m = 2 * C * M_L * 2 ** L * (P - 1) * Q / G
-    return s2t + s2m
+    return 6 * C * M_L * M_L * 2 ** L * (P - 1) / G
 
 
 class ClockSampler:
@@ -327,8 +326,8 @@ def run_fmmfft(args, rank, world, local_rank):
     if rank != 0:
         return
     peaks = load_peaks()
-    fl = near_up_flops(N, P, B, Q, M_L, G)
-    t_near = stages.get("near_up", float("nan")) * 1e-3
+    fl = s2t_flops(N, P, M_L, G)
+    t_near = stages.get("s2t", float("nan")) * 1e-3
     sm_max = peaks.get("sm_max_mhz", 1965.0)
     if prec == "c64":
         peak = 148 * 128 * 2 * sm_max * 1e6 / 1e12            # FP32 FMA lanes x 2 flops x max clock
@@ -344,7 +343,7 @@ def run_fmmfft(args, rank, world, local_rank):
         "config": {"workload": workload, "desc": desc, "N": N, "P": P, "G": G, "B": B, "Q": Q, "M_L": M_L,
                    "L": info["L"], "precision": prec, "l2": "flushed (256 MiB write between steps, outside events)",
                    "parseval_rel_dev": parseval},
-        "roofline": {"kernel": "k_near_up (S2T + S2M)", "bound": "alu", "achieved": achieved, "peak": peak,
+        "roofline": {"kernel": "k_near_up (S2T, side stream, concurrent with the far field)", "bound": "alu", "achieved": achieved, "peak": peak,
                      "unit": "TFLOP/s", "frac": achieved / peak, "traffic": load_traffic(workload, G),
                      "algorithmic_flops_per_launch": fl, "avg_launch_ms": t_near * 1e3,
                      "peak_basis": f"148 SMs x {'128 FP32' if prec == 'c64' else '64 FP64'} FMA/clk x 2 x {sm_max} MHz"},

@@ -121,7 +121,9 @@ FMMFFT_API fmmfft_status_t fmmfft_get_info(fmmfft_plan_t plan, fmmfft_info_t* in
 
 /* Per-stage device times (ms) of the LAST execute of a plan created with
  * FMMFFT_FLAG_PROFILE (else INVALID_VALUE); synchronises that execute's stream. Stage i's
- * name is fmmfft_stage_name(i). n = capacity of ms[]; returns the count in *n_out. */
+ * name is fmmfft_stage_name(i): comm_S, s2m, m2m, comm_M, top, down, post_pfft, a2a, mfft —
+ * consecutive intervals of the main stream — and s2t, the near field on the side stream that
+ * overlaps s2m..down. n = capacity of ms[]; returns the count in *n_out. */
 FMMFFT_API fmmfft_status_t fmmfft_stage_times(fmmfft_plan_t plan, float* ms, int n, int* n_out);
 FMMFFT_API const char* fmmfft_stage_name(int i);
 

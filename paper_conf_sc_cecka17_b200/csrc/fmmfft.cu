@@ -100,9 +100,10 @@ static double lagr(const std::vector<double>& z, int i, double t) {   // l_i(t) 
 static double cotpi(double x) { return std::cos(M_PI * x) / std::sin(M_PI * x); }  // cot(pi x)
 
 // ------------------------------------------------------------------ plan
+// Stages on the main stream (consecutive events), plus S2T on the side stream (its own pair).
 enum Stage { ST_COMM_S, ST_NEAR, ST_M2M, ST_COMM_M, ST_TOP, ST_DOWN, ST_PFFT, ST_A2A, ST_MFFT, ST_COUNT };
-static const char* kStageNames[ST_COUNT] = {"comm_S", "near_up", "m2m", "comm_M", "top",
-                                            "down", "post_pfft", "a2a", "mfft"};
+static const char* kStageNames[ST_COUNT + 1] = {"comm_S", "s2m", "m2m", "comm_M", "top",
+                                                "down", "post_pfft", "a2a", "mfft", "s2t"};
 
 struct RankBufs {
     int g = 0;
@@ -151,6 +152,9 @@ struct fmmfft_plan_s {
     size_t ws_bytes = 0;
     int kernels = 0;
     cudaEvent_t ev[fmmfft::ST_COUNT + 1] = {};
+    cudaEvent_t ev_s2t[2] = {};      // S2T on the side stream (profiling)
+    cudaEvent_t fork = nullptr, join = nullptr;   // side-stream fork / join
+    cudaStream_t side = nullptr;     // S2T runs here, concurrently with the far field
     bool have_times = false;
     bool use_graph = true;
     cudaStream_t cap_stream = nullptr;
@@ -310,6 +314,11 @@ static void destroy_plan(fmmfft_plan_s* p) {
     for (void* a : p->allocs) cudaFree(a);
     for (auto& ev : p->ev)
         if (ev) cudaEventDestroy(ev);
+    for (auto& ev : p->ev_s2t)
+        if (ev) cudaEventDestroy(ev);
+    if (p->fork) cudaEventDestroy(p->fork);
+    if (p->join) cudaEventDestroy(p->join);
+    if (p->side) cudaStreamDestroy(p->side);
     if (p->cap_stream) cudaStreamDestroy(p->cap_stream);
     delete p;
 }
@@ -334,6 +343,7 @@ static fmmfft_status_t init_kernel_attrs() {
         auto per_pc = [&](auto pc) {
             constexpr int PCv = decltype(pc)::value;
             set((const void*)k_near_up<R, IB, PCv>);
+            set((const void*)k_s2m<R, PCv>);
             if constexpr (PCv <= (sizeof(R) == 4 ? 16 : 8)) {
                 set((const void*)k_up<R, PCv>);
                 set((const void*)k_down<R, 2, PCv>);
@@ -352,6 +362,10 @@ static fmmfft_status_t init_kernel_attrs() {
             }
         };
         for (int pc = 2; pc <= (sizeof(R) == 4 ? 32 : 16); pc *= 2) dispatch<2, 4, 8, 16, 32>(pc, per_pc);
+        if constexpr (sizeof(R) == 4) {
+            set((const void*)k_tree_pq<16, 512, 8>);
+            set((const void*)k_tree_pq<8, 512, 8>);
+        }
         set((const void*)k_tree_p<R, 1>);
         set((const void*)k_tree_p<R, 2>);
         set((const void*)k_tree_p<R, 4>);
@@ -432,8 +446,36 @@ struct Exec {
         return FMMFFT_SUCCESS;
     }
 
-    // ---- near_up: S2T + S2M
+    // record a stage-boundary-style event on an arbitrary stream (S2T's own pair)
+    fmmfft_status_t mark_on(cudaEvent_t e, cudaStream_t st) {
+        if (p->flags & FMMFFT_FLAG_PROFILE)
+            CUDA_TRY(cudaEventRecordWithFlags(e, st, p->use_graph ? cudaEventRecordExternal : cudaEventRecordDefault));
+        return FMMFFT_SUCCESS;
+    }
+
+    // ---- near field: S2M on the main stream; S2T forked onto the side stream (joined before
+    // post_pfft), so the far field and the near field run concurrently
     fmmfft_status_t near_up() {
+        fmmfft_status_t st;
+        // fork: the side stream starts after the S halo is in place
+        CUDA_TRY(cudaEventRecord(p->fork, s));
+        CUDA_TRY(cudaStreamWaitEvent(p->side, p->fork, 0));
+        const int PCs = std::min(p->P, sizeof(R) == 4 ? 32 : 16);
+        for (RankBufs& rb : p->ranks) {
+            const C* S = in[p->virt ? rb.g : 0];
+            const int Qp = (p->Q + 3) / 4 * 4;
+            const size_t smem = (size_t)p->M_L * PCs * sizeof(C) + (size_t)Qp * p->M_L * sizeof(R);
+            const dim3 grid((unsigned)p->nb, (unsigned)(p->P / PCs));
+            dispatch<2, 4, 8, 16, 32>(PCs, [&](auto pc) {
+                constexpr int PCv = decltype(pc)::value;
+                if constexpr (!(sizeof(R) == 8 && PCv > 16))
+                    k_s2m<R, PCv><<<grid, PCv * (Qp / 4), smem, s>>>(S, interior(rb.Mpad[p->L]), (const R*)p->s2m, p->P,
+                                                                     p->M_L, p->Q);
+            });
+            LAUNCH_CHECK();
+        }
+        // S2T on the side stream
+        if ((st = mark_on(p->ev_s2t[0], p->side))) return st;
         const int PC_ = p->PCn, nib = p->M_L / IB;
         const int threads = PC_ * nib;
         const int npc = p->P / PC_;
@@ -451,13 +493,21 @@ struct Exec {
                 constexpr int PCv = decltype(pc)::value;
                 if constexpr (sizeof(R) == 8 && PCv > 16) return;
                 else
-                    k_near_up<R, IB, PCv><<<grid, threads, smem, s>>>(S, hl, hr, (C*)rb.Tn, interior(rb.Mpad[p->L]),
-                                                                      (const R*)p->s2t, p->s2t_chunk, (const R*)p->s2m,
-                                                                      p->P, p->M_L, p->Q, p->nb, bpc);
+                    k_near_up<R, IB, PCv><<<grid, threads, smem, p->side>>>(S, hl, hr, (C*)rb.Tn, nullptr,
+                                                                            (const R*)p->s2t, p->s2t_chunk, (const R*)p->s2m,
+                                                                            p->P, p->M_L, p->Q, p->nb, bpc);
             };
             dispatch<2, 4, 8, 16, 32>(PC_, go);
             LAUNCH_CHECK();
         }
+        if ((st = mark_on(p->ev_s2t[1], p->side))) return st;
+        CUDA_TRY(cudaEventRecord(p->join, p->side));
+        return FMMFFT_SUCCESS;
+    }
+
+    // join the side stream (S2T) before the near and far fields are combined
+    fmmfft_status_t join_near() {
+        CUDA_TRY(cudaStreamWaitEvent(s, p->join, 0));
         return FMMFFT_SUCCESS;
     }
 
@@ -500,13 +550,24 @@ struct Exec {
             a.r = rb.r;
             a.L = p->L;
             a.B = p->B;
+            const int tabB = ((1 << p->B) - 3) * p->Q * p->Q;
+            // complex64 with Q = 16 or 8 and <= 8 boxes per thread group: register-blocked kernel
+            if constexpr (sizeof(R) == 4) {
+                const int ngrp = 512 / p->Q;
+                if ((p->Q == 16 || p->Q == 8) && (1LL << p->L) <= 8LL * ngrp) {
+                    const size_t smem = tree_p_smem(p, 512) + ((size_t)p->Q << p->L) * sizeof(C);   // + scratch
+                    if (p->Q == 16) k_tree_pq<16, 512, 8><<<p->P - 1, 512, smem, s>>>(a, (const float*)p->m2m, p->P, tabB);
+                    else            k_tree_pq<8, 512, 8><<<p->P - 1, 512, smem, s>>>(a, (const float*)p->m2m, p->P, tabB);
+                    LAUNCH_CHECK();
+                    continue;
+                }
+            }
             const int threads = sizeof(R) == 4 ? 1024 : 512;
             const int maxo = (int)((((long long)p->Q << p->L) + threads - 1) / threads);
             const size_t smem = tree_p_smem(p, threads);
             dispatch<1, 2, 4, 8>(maxo <= 1 ? 1 : maxo <= 2 ? 2 : maxo <= 4 ? 4 : 8, [&](auto mo) {
                 constexpr int MO = decltype(mo)::value;
-                k_tree_p<R, MO><<<p->P - 1, threads, smem, s>>>(a, (const R*)p->m2m, p->P, p->Q,
-                                                                ((1 << p->B) - 3) * p->Q * p->Q);
+                k_tree_p<R, MO><<<p->P - 1, threads, smem, s>>>(a, (const R*)p->m2m, p->P, p->Q, tabB);
             });
             LAUNCH_CHECK();
         }
@@ -696,14 +757,16 @@ struct Exec {
     fmmfft_status_t post_pfft() {
         const int MS = std::min(p->M_L, std::max(1, TILE / p->P));
         const int threads = std::min(sizeof(R) == 4 ? 1024 : 512, std::max(32, MS * p->P / 8));
-        const size_t smem = (size_t)MS * (p->P + 1) * sizeof(C) + (size_t)p->P * sizeof(C) + (size_t)p->Q * MS * sizeof(R);
+        size_t smem = (size_t)MS * (p->P + 1) * sizeof(C) + (size_t)p->P * sizeof(C) + (size_t)p->Q * MS * sizeof(R);
+        const int stage_L = smem + (size_t)p->Q * p->P * sizeof(C) <= 160 * 1024;   // stage L^L of the box
+        if (stage_L) smem += (size_t)p->Q * p->P * sizeof(C);
         const int blocks = p->nb * (p->M_L / MS);
         for (RankBufs& rb : p->ranks) {
             dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 11>(ilog2(p->P), [&](auto lp) {
                 constexpr int LP = decltype(lp)::value;
                 k_post_pfft<R, LP><<<blocks, threads, smem, s>>>((const C*)rb.Tn, (const C*)rb.Lloc[p->L], (const C*)rb.r,
                                                                 (const C*)p->rho, (const R*)p->s2m, (C*)rb.W,
-                                                                ilog2(p->M_L), p->Q, ilog2(MS), (int)p->Mg);
+                                                                ilog2(p->M_L), p->Q, ilog2(MS), (int)p->Mg, stage_L);
             });
             LAUNCH_CHECK();
         }
@@ -777,6 +840,7 @@ struct Exec {
         STEP(ST_COMM_M, comm_M())
         STEP(ST_TOP, top())
         STEP(ST_DOWN, down())
+        if ((st = join_near())) return st;
         STEP(ST_PFFT, post_pfft())
         STEP(ST_A2A, a2a())
         STEP(ST_MFFT, mfft())
@@ -853,7 +917,7 @@ extern "C" {
 
 const char* fmmfft_last_error(void) { return g_last_error.c_str(); }
 const char* fmmfft_version(void) { return "fmmfft-b200 0.2 (sm_100a)"; }
-const char* fmmfft_stage_name(int i) { return (i >= 0 && i < ST_COUNT) ? kStageNames[i] : ""; }
+const char* fmmfft_stage_name(int i) { return (i >= 0 && i <= ST_COUNT) ? kStageNames[i] : ""; }
 
 fmmfft_status_t fmmfft_get_unique_id(unsigned char id[128]) {
     if (!id) return fail(FMMFFT_INVALID_VALUE, "id is NULL");
@@ -937,7 +1001,8 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
         const int threads = precision == FMMFFT_C64 ? 1024 : 512;
         int optin = 0;
         cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-        p->tree_p = (G == 1) && ((long long)Q << L) <= 8LL * threads && tree_p_smem(p, threads) <= (size_t)optin;
+        const size_t scratch = ((size_t)Q << L) * p->esz;
+        p->tree_p = (G == 1) && ((long long)Q << L) <= 8LL * threads && tree_p_smem(p, threads) + scratch <= (size_t)optin;
         if (const char* e = getenv("FMMFFT_TREE")) p->tree_p = p->tree_p && e[0] == 'p';
     }
     const char* g_env = getenv("FMMFFT_NO_GRAPH");
@@ -960,7 +1025,14 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
     }
     if (!st) {
         cudaError_t e = cudaStreamCreateWithFlags(&p->cap_stream, cudaStreamNonBlocking);
-        if (e != cudaSuccess) st = fail(FMMFFT_CUDA_ERROR, "cudaStreamCreate: %s", cudaGetErrorString(e));
+        if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&p->side, cudaStreamNonBlocking);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->fork, cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->join, cudaEventDisableTiming);
+        if (e == cudaSuccess && (flags & FMMFFT_FLAG_PROFILE)) {
+            e = cudaEventCreate(&p->ev_s2t[0]);
+            if (e == cudaSuccess) e = cudaEventCreate(&p->ev_s2t[1]);
+        }
+        if (e != cudaSuccess) st = fail(FMMFFT_CUDA_ERROR, "stream/event setup: %s", cudaGetErrorString(e));
     }
     if (!st) {
         cudaError_t e = cudaDeviceSynchronize();
@@ -1021,7 +1093,7 @@ fmmfft_status_t fmmfft_get_info(fmmfft_plan_t p, fmmfft_info_t* info) {
     if (!p || !info) return fail(FMMFFT_INVALID_VALUE, "NULL argument");
     info->N = p->N; info->P = p->P; info->G = p->G; info->B = p->B; info->Q = p->Q; info->M_L = p->M_L;
     info->L = p->L; info->precision = p->prec; info->M = p->M; info->level_gather = p->lg;
-    info->n_stages = ST_COUNT; info->workspace_bytes = p->ws_bytes; info->kernels_per_execute = p->kernels;
+    info->n_stages = ST_COUNT + 1; info->workspace_bytes = p->ws_bytes; info->kernels_per_execute = p->kernels;
     return FMMFFT_SUCCESS;
 }
 
@@ -1029,8 +1101,9 @@ fmmfft_status_t fmmfft_stage_times(fmmfft_plan_t p, float* ms, int n, int* n_out
     if (!p || !ms || !n_out) return fail(FMMFFT_INVALID_VALUE, "NULL argument");
     if (!(p->flags & FMMFFT_FLAG_PROFILE) || !p->have_times) return fail(FMMFFT_INVALID_VALUE, "plan not profiled / not executed");
     CUDA_TRY(cudaEventSynchronize(p->ev[ST_COUNT]));
-    const int k = std::min(n, (int)ST_COUNT);
-    for (int i = 0; i < k; ++i) CUDA_TRY(cudaEventElapsedTime(&ms[i], p->ev[i], p->ev[i + 1]));
+    const int k = std::min(n, (int)ST_COUNT + 1);
+    for (int i = 0; i < k && i < ST_COUNT; ++i) CUDA_TRY(cudaEventElapsedTime(&ms[i], p->ev[i], p->ev[i + 1]));
+    if (k > ST_COUNT) CUDA_TRY(cudaEventElapsedTime(&ms[ST_COUNT], p->ev_s2t[0], p->ev_s2t[1]));
     *n_out = k;
     return FMMFFT_SUCCESS;
 }

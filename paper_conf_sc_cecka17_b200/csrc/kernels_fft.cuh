@@ -139,29 +139,32 @@ template <typename R, int LP>
 __global__ void __launch_bounds__(sizeof(R) == 4 ? 1024 : 512)
 k_post_pfft(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2<R>* __restrict__ r,
             const C2<R>* __restrict__ rho, const R* __restrict__ s2m, C2<R>* __restrict__ W,
-            int lML, int Q, int lMS, int Mg) {
+            int lML, int Q, int lMS, int Mg, int stage_L) {
     using C = C2<R>;
     constexpr int P = 1 << LP, LD = P + 1;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     const int MS = 1 << lMS, M_L = 1 << lML;
     C* tile = reinterpret_cast<C*>(smem_raw);                    // [MS][P + 1]
     C* tw = tile + MS * LD;                                       // [P]
-    R* s2m_sm = reinterpret_cast<R*>(tw + P);                    // [Q][MS]
+    C* Lsm = tw + P;                                              // [Q][P]   L^L of box b (if staged)
+    R* s2m_sm = reinterpret_cast<R*>(Lsm + (stage_L ? Q * P : 0)); // [Q][MS]
     const int tid = threadIdx.x, nthr = blockDim.x;
     const int lnsub = lML - lMS;
     const int b = blockIdx.x >> lnsub, m0 = (blockIdx.x & ((1 << lnsub) - 1)) << lMS;
 
     const C* src = Tn + (((size_t)b << lML) + m0) * P;
     for (int idx = tid; idx < (MS << LP); idx += nthr) cp_async_elem(tile + (idx >> LP) * LD + (idx & (P - 1)), src + idx);
+    const C* Lb = LL + (size_t)b * Q * P;
+    if (stage_L)
+        for (int idx = tid; idx < Q * P; idx += nthr) cp_async_elem(Lsm + idx, Lb + idx);
     for (int idx = tid; idx < Q * MS; idx += nthr) cp_async_elem(s2m_sm + idx, s2m + (idx >> lMS) * M_L + m0 + (idx & (MS - 1)));
     fill_twiddles<R>(tw, LP);
     cp_async_wait_all();
     __syncthreads();
 
-    // L2T + POST: thread owns one p and a group of MG consecutive m (L^L loaded once per q).
+    // L2T + POST: thread owns one p and a group of MG consecutive m (L^L read once per q).
     constexpr int MG = 8;
     const int ngrp = (MS + MG - 1) / MG;
-    const C* Lb = LL + (size_t)b * Q * P;
     for (int idx = tid; idx < P * ngrp; idx += nthr) {
         const int p = idx & (P - 1), g = idx >> LP;
         if (p == 0) continue;                                      // C_0 = I (R1)
@@ -169,7 +172,7 @@ k_post_pfft(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2
 #pragma unroll
         for (int u = 0; u < MG; ++u) acc[u] = zero<C>();
         for (int q = 0; q < Q; ++q) {
-            const C l = ldg_c(Lb + q * P + p);
+            const C l = stage_L ? Lsm[q * P + p] : ldg_c(Lb + q * P + p);
 #pragma unroll
             for (int u = 0; u < MG; ++u)
                 if (g * MG + u < MS) rfma(acc[u], s2m_sm[q * MS + g * MG + u], l);

@@ -23,3 +23,17 @@ for r in top:
     st = {k: int(r[I[k]] or 0) for k in hdr if k.startswith("stall_") and "Not Issued" not in k}
     main = sorted(st.items(), key=lambda kv: -kv[1])[:2]
     print(f"{int(r[I['# Samples']]) / tot_s:6.1%}  {r[I['Source']].strip()[:60]:60s} {main}")
+
+
+def stall_totals(path):
+    rows = list(csv.reader(open(path)))
+    hdr = rows[1]
+    I = {h: i for i, h in enumerate(hdr)}
+    data = [r for r in rows[2:] if len(r) == len(hdr) and r[0] != "Address"]
+    tot = Counter()
+    for r in data:
+        for k in hdr:
+            if k.startswith("stall_") and "Not Issued" not in k:
+                tot[k] += int(r[I[k]] or 0)
+    s = sum(tot.values()) or 1
+    return ", ".join(f"{k[6:]}:{v / s:.0%}" for k, v in tot.most_common(8))

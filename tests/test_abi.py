@@ -69,8 +69,8 @@ def test_null_arguments(L):
 
 
 def test_stage_names(L):
-    names = [L.lib.fmmfft_stage_name(i).decode() for i in range(9)]
-    assert names == ["comm_S", "near_up", "m2m", "comm_M", "top", "down", "post_pfft", "a2a", "mfft"]
+    names = [L.lib.fmmfft_stage_name(i).decode() for i in range(10)]
+    assert names == ["comm_S", "s2m", "m2m", "comm_M", "top", "down", "post_pfft", "a2a", "mfft", "s2t"]
     assert L.lib.fmmfft_stage_name(99) == b""
 
 

@@ -184,8 +184,8 @@ def test_profile_stage_times(F):
     x = torch.from_numpy(SI.complex_uniform(0, 1 << 20, dtype=np.complex64)).cuda()
     plan(x)
     t = plan.stage_times()
-    assert list(t) == ["comm_S", "near_up", "m2m", "comm_M", "top", "down", "post_pfft", "a2a", "mfft"]
-    assert all(v >= 0 for v in t.values()) and t["near_up"] > 0
+    assert list(t) == ["comm_S", "s2m", "m2m", "comm_M", "top", "down", "post_pfft", "a2a", "mfft", "s2t"]
+    assert all(v >= 0 for v in t.values()) and t["s2t"] > 0
     assert plan.info["kernels_per_execute"] >= 4
 
 
