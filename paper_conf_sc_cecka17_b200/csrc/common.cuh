@@ -12,9 +12,12 @@ template <> struct cplx<float> { using type = float2; };
 template <> struct cplx<double> { using type = double2; };
 template <typename R> using C2 = typename cplx<R>::type;
 
-__device__ __forceinline__ float2 cadd(float2 a, float2 b) { return make_float2(a.x + b.x, a.y + b.y); }
+// Blackwell packs two fp32 lanes per instruction (FADD2 / FMUL2 / FFMA2, PTX .f32x2): a complex
+// value is one float2 register pair, and a real operator entry times complex data is a single
+// FFMA2 with the scalar broadcast — the FMM's whole arithmetic shape.
+__device__ __forceinline__ float2 cadd(float2 a, float2 b) { return __fadd2_rn(a, b); }
 __device__ __forceinline__ double2 cadd(double2 a, double2 b) { return make_double2(a.x + b.x, a.y + b.y); }
-__device__ __forceinline__ float2 csub(float2 a, float2 b) { return make_float2(a.x - b.x, a.y - b.y); }
+__device__ __forceinline__ float2 csub(float2 a, float2 b) { return __fadd2_rn(a, make_float2(-b.x, -b.y)); }
 __device__ __forceinline__ double2 csub(double2 a, double2 b) { return make_double2(a.x - b.x, a.y - b.y); }
 __device__ __forceinline__ float2 cmul(float2 a, float2 b) {
     return make_float2(fmaf(a.x, b.x, -a.y * b.y), fmaf(a.x, b.y, a.y * b.x));
@@ -23,7 +26,7 @@ __device__ __forceinline__ double2 cmul(double2 a, double2 b) {
     return make_double2(fma(a.x, b.x, -a.y * b.y), fma(a.x, b.y, a.y * b.x));
 }
 // a += k * b for real k (the FMM operators are real)
-__device__ __forceinline__ void rfma(float2& a, float k, float2 b) { a.x = fmaf(k, b.x, a.x); a.y = fmaf(k, b.y, a.y); }
+__device__ __forceinline__ void rfma(float2& a, float k, float2 b) { a = __ffma2_rn(make_float2(k, k), b, a); }
 __device__ __forceinline__ void rfma(double2& a, double k, double2 b) { a.x = fma(k, b.x, a.x); a.y = fma(k, b.y, a.y); }
 __device__ __forceinline__ float2 czero(float2) { return make_float2(0.f, 0.f); }
 __device__ __forceinline__ double2 czero(double2) { return make_double2(0.0, 0.0); }
