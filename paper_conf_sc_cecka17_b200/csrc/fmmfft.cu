@@ -35,6 +35,7 @@
 #include "common.cuh"
 #include "kernels_fft.cuh"
 #include "kernels_fmm.cuh"
+#include "kernel_s2t_tc.cuh"
 #include "nccl_loader.hpp"
 
 namespace fmmfft {
@@ -109,6 +110,7 @@ struct RankBufs {
     int g = 0;
     void* Tn = nullptr;      // [nb][M_L][P]   S2T output (T_near)
     void* tmp = nullptr;     // M-FFT ping-pong buffer
+    void* Sp = nullptr;      // S'[p][b][m]: p-major copy of the input for the tensor-core S2T
     void* W = nullptr;       // [k2][Mg]       P-FFT output = all-to-all send buffer
     void* Rcv = nullptr;     // all-to-all receive buffer (G > 1)
     void* haloL = nullptr;   // S box -1  (G > 1)
@@ -147,6 +149,9 @@ struct fmmfft_plan_s {
     std::vector<void*> m2l;          // by level
     std::vector<void*> m2l_pmaj;     // p-major copies for the fused per-p tree (G = 1), by level
     bool tree_p = false;             // use k_tree_p for the far field
+    bool tree_phased = false;        // ... as up / all-levels M2L / L2L-chain launches (FMMFFT_TREE=p) (k_tree_pq<.., false>, k_m2l_flat, k_tree_dn)
+    bool s2t_tc = false;             // S2T on tcgen05 (k_s2t_tc): complex64, M_L = 64, nb % 64 == 0
+    void* toep = nullptr;            // its Toeplitz hi/lo operand table
     std::vector<fmmfft::RankBufs> ranks;
     std::vector<int> radices;        // M-FFT passes
     size_t ws_bytes = 0;
@@ -154,6 +159,7 @@ struct fmmfft_plan_s {
     cudaEvent_t ev[fmmfft::ST_COUNT + 1] = {};
     cudaEvent_t ev_s2t[2] = {};      // S2T on the side stream (profiling)
     cudaEvent_t fork = nullptr, join = nullptr;   // side-stream fork / join
+    cudaEvent_t fork2 = nullptr;     // S' ready (tensor-core S2T)
     cudaStream_t side = nullptr;     // S2T runs here, concurrently with the far field
     bool have_times = false;
     bool use_graph = true;
@@ -249,6 +255,38 @@ static fmmfft_status_t build_tables(fmmfft_plan_s* p) {
             if ((st = upload<R>(p, &p->m2l_pmaj[lev], tp))) return st;
         }
     }
+    // tensor-core S2T operand: Toep_p[i][k] = S2T_{p, (k - 64) - i}, split into tf32 hi + lo,
+    // in the UMMA K-major core-matrix layout [p][chunk][hi/lo][k4][r8][8][4] (kernel_s2t_tc.cuh)
+    if (p->s2t_tc) {
+        auto tf32 = [](double v) {                     // round to nearest (ties away), tf32 precision
+            float f = (float)v;
+            uint32_t u;
+            memcpy(&u, &f, 4);
+            u = (u + 0x1000u) & 0xFFFFE000u;
+            memcpy(&f, &u, 4);
+            return f;
+        };
+        std::vector<float> tb((size_t)P * S2TC_TAB_FLOATS_PER_P, 0.f);
+        const int half = 64 * S2TC_CHUNK_K;                // floats of one of hi / lo per chunk
+        for (int pp = 1; pp < P; ++pp)
+            for (int c = 0; c < S2TC_NCHUNK; ++c)
+                for (int k4 = 0; k4 < S2TC_CHUNK_K / 4; ++k4)
+                    for (int i = 0; i < 64; ++i)
+                        for (int kk = 0; kk < 4; ++kk) {
+                            const int k = S2TC_CHUNK_K * c + 4 * k4 + kk;
+                            const long long d = (long long)(k - 64) - i;
+                            const double v = cotpi((double)(pp + (long long)P * d) / (double)N);
+                            const float hi = tf32(v);
+                            const float lo = tf32(v - (double)hi);
+                            const size_t base = (size_t)pp * S2TC_TAB_FLOATS_PER_P + (size_t)c * 2 * half;
+                            const size_t e = ((size_t)(k4 * 8 + (i >> 3)) * 8 + (i & 7)) * 4 + kk;
+                            tb[base + e] = hi;
+                            tb[base + half + e] = lo;
+                        }
+        fmmfft_status_t st2 = dalloc(p, &p->toep, tb.size() * sizeof(float));
+        if (st2) return st2;
+        CUDA_TRY(cudaMemcpy(p->toep, tb.data(), tb.size() * sizeof(float), cudaMemcpyHostToDevice));
+    }
     // rho_p = exp(-i pi p/P) sin(pi p/P) / M, interleaved complex; rho_0 unused
     std::vector<double> rho(2 * (size_t)P);
     for (int pp = 0; pp < P; ++pp) {
@@ -282,6 +320,7 @@ static fmmfft_status_t alloc_rank(fmmfft_plan_s* p, RankBufs& rb) {
     if ((st = dalloc(p, &rb.Tn, n_local * e))) return st;
     if ((st = dalloc(p, &rb.W, n_local * e))) return st;
     if ((st = dalloc(p, &rb.tmp, n_local * e))) return st;
+    if (p->s2t_tc && (st = dalloc(p, &rb.Sp, n_local * e))) return st;
     if (p->G > 1) {
         if ((st = dalloc(p, &rb.Rcv, n_local * e))) return st;
         if ((st = dalloc(p, &rb.haloL, (size_t)p->M_L * p->P * e))) return st;
@@ -318,6 +357,7 @@ static void destroy_plan(fmmfft_plan_s* p) {
         if (ev) cudaEventDestroy(ev);
     if (p->fork) cudaEventDestroy(p->fork);
     if (p->join) cudaEventDestroy(p->join);
+    if (p->fork2) cudaEventDestroy(p->fork2);
     if (p->side) cudaStreamDestroy(p->side);
     if (p->cap_stream) cudaStreamDestroy(p->cap_stream);
     delete p;
@@ -346,10 +386,7 @@ static fmmfft_status_t init_kernel_attrs() {
             set((const void*)k_s2m<R, PCv>);
             if constexpr (PCv <= (sizeof(R) == 4 ? 16 : 8)) {
                 set((const void*)k_up<R, PCv>);
-                set((const void*)k_down<R, 2, PCv>);
-                set((const void*)k_down<R, 4, PCv>);
-                set((const void*)k_down<R, 8, PCv>);
-                set((const void*)k_down<R, 16, PCv>);
+                set((const void*)k_m2l_flat<R, 8, PCv>);
                 set((const void*)k_base<R, 4, PCv>);
                 set((const void*)k_base<R, 8, PCv>);
                 set((const void*)k_base<R, 16, PCv>);
@@ -364,8 +401,13 @@ static fmmfft_status_t init_kernel_attrs() {
         for (int pc = 2; pc <= (sizeof(R) == 4 ? 32 : 16); pc *= 2) dispatch<2, 4, 8, 16, 32>(pc, per_pc);
         if constexpr (sizeof(R) == 4) {
             set((const void*)k_tree_pq<16, 512, 8>);
+            set((const void*)k_tree_pq<16, 512, 8, false>);
+            set((const void*)k_tree_pq<8, 512, 8, false>);
+            set((const void*)k_tree_dn<16, 512>);
+            set((const void*)k_tree_dn<8, 512>);
             set((const void*)k_tree_pq<8, 512, 8>);
         }
+        if constexpr (sizeof(R) == 4) set((const void*)k_s2t_tc);
         set((const void*)k_tree_p<R, 1>);
         set((const void*)k_tree_p<R, 2>);
         set((const void*)k_tree_p<R, 4>);
@@ -470,12 +512,32 @@ struct Exec {
                 constexpr int PCv = decltype(pc)::value;
                 if constexpr (!(sizeof(R) == 8 && PCv > 16))
                     k_s2m<R, PCv><<<grid, PCv * (Qp / 4), smem, s>>>(S, interior(rb.Mpad[p->L]), (const R*)p->s2m, p->P,
-                                                                     p->M_L, p->Q);
+                                                                     p->M_L, p->Q, (C*)rb.Sp, p->nb);
             });
             LAUNCH_CHECK();
         }
         // S2T on the side stream
         if ((st = mark_on(p->ev_s2t[0], p->side))) return st;
+        if constexpr (sizeof(R) == 4) {
+            if (p->s2t_tc) {                                   // tensor cores (tcgen05, 3xTF32)
+                CUDA_TRY(cudaEventRecord(p->fork2, s));             // needs S' from k_s2m
+                CUDA_TRY(cudaStreamWaitEvent(p->side, p->fork2, 0));
+                if ((st = mark_on(p->ev_s2t[0], p->side))) return st;
+                for (RankBufs& rb : p->ranks) {
+                    const C* S = in[p->virt ? rb.g : 0];
+                    const size_t box = (size_t)p->M_L * p->P;
+                    const C* hl = p->G == 1 ? S + (size_t)(p->nb - 1) * box : (const C*)rb.haloL;
+                    const C* hr = p->G == 1 ? S : (const C*)rb.haloR;
+                    const dim3 grid((unsigned)(p->nb / S2TC_BOXES), (unsigned)p->P);
+                    k_s2t_tc<<<grid, 256, s2tc_smem_bytes(), p->side>>>((const C*)rb.Sp, S, hl, hr, (C*)rb.Tn,
+                                                                         (const float*)p->toep, p->P, p->nb, p->G);
+                    LAUNCH_CHECK();
+                }
+                if ((st = mark_on(p->ev_s2t[1], p->side))) return st;
+                CUDA_TRY(cudaEventRecord(p->join, p->side));
+                return FMMFFT_SUCCESS;
+            }
+        }
         const int PC_ = p->PCn, nib = p->M_L / IB;
         const int threads = PC_ * nib;
         const int npc = p->P / PC_;
@@ -554,6 +616,43 @@ struct Exec {
             // complex64 with Q = 16 or 8 and <= 8 boxes per thread group: register-blocked kernel
             if constexpr (sizeof(R) == 4) {
                 const int ngrp = 512 / p->Q;
+                if ((p->Q == 16 || p->Q == 8) && (1LL << p->L) <= 8LL * ngrp && p->tree_phased) {
+                    // (1) M2M + M2L-B + REDUCE per FMM, (2) all levels' M2L in one wide launch,
+                    // (3) the L2L chain per FMM
+                    const size_t smem1 = tree_p_smem(p, 512);
+                    if (p->Q == 16) k_tree_pq<16, 512, 8, false><<<p->P - 1, 512, smem1, s>>>(a, (const float*)p->m2m, p->P, tabB);
+                    else            k_tree_pq<8, 512, 8, false><<<p->P - 1, 512, smem1, s>>>(a, (const float*)p->m2m, p->P, tabB);
+                    LAUNCH_CHECK();
+                    if (p->L > p->B) {
+                        M2LFlat f{};
+                        constexpr int BR = 8;
+                        int tiles = 0;
+                        for (int lev = p->B + 1; lev <= p->L; ++lev) {
+                            f.src[lev] = interior(rb.Mpad[lev]);
+                            f.out[lev] = rb.Lloc[lev];
+                            f.tab[lev] = p->m2l[lev];
+                            f.tile0[lev] = tiles;
+                            tiles += ((1 << lev) + BR - 1) / BR;
+                        }
+                        f.tile0[p->L + 1] = tiles;
+                        f.lmin = p->B + 1;
+                        f.lmax = p->L;
+                        const int PC_ = p->PCd;
+                        const size_t smem2 = (size_t)(BR + 4 + BR / 2) * p->Q * PC_ * sizeof(C) + (size_t)p->m2l_chunk * sizeof(R) +
+                                             (size_t)2 * p->Q * p->Q * sizeof(R) + (BR + 4) * sizeof(int);
+                        const dim3 grid((unsigned)tiles, (unsigned)(p->P / PC_));
+                        with_pcd([&](auto pc) {
+                            constexpr int PCv = decltype(pc)::value;
+                            k_m2l_flat<R, BR, PCv><<<grid, PCv * p->Q, smem2, s>>>(f, p->m2l_chunk, (const R*)p->m2m, p->P, p->Q);
+                        });
+                        LAUNCH_CHECK();
+                        const size_t smem3 = (((size_t)2 << p->L) - ((size_t)1 << p->B)) * p->Q * sizeof(C) + (size_t)2 * p->Q * p->Q * sizeof(R);
+                        if (p->Q == 16) k_tree_dn<16, 512><<<p->P - 1, 512, smem3, s>>>(a, (const float*)p->m2m, p->P);
+                        else            k_tree_dn<8, 512><<<p->P - 1, 512, smem3, s>>>(a, (const float*)p->m2m, p->P);
+                        LAUNCH_CHECK();
+                    }
+                    continue;
+                }
                 if ((p->Q == 16 || p->Q == 8) && (1LL << p->L) <= 8LL * ngrp) {
                     const size_t smem = tree_p_smem(p, 512) + ((size_t)p->Q << p->L) * sizeof(C);   // + scratch
                     if (p->Q == 16) k_tree_pq<16, 512, 8><<<p->P - 1, 512, smem, s>>>(a, (const float*)p->m2m, p->P, tabB);
@@ -621,31 +720,6 @@ struct Exec {
         }
         NCCL_TRY(n.GroupEnd());
         NCCL_TRY(n.AllGather(interior(rb.Mpad[p->lg]), rb.Mfull[p->lg], 2 * nlg * QPc, nt(), g_comm.comm, s));
-        return FMMFFT_SUCCESS;
-    }
-
-    // M2L + L2L for one interaction-list level (l > B)
-    fmmfft_status_t launch_down(const C* src, long long src_base, int src_mod, const C* parent, long long par_base,
-                                C* outp, long long tgt_base, int ntg, int lev) {
-        const int PC_ = p->PCd;
-        const int npc = p->P / PC_;
-        // the table slice (4 Q^2 PC) is loaded once per CTA: prefer 16 targets per CTA, fewer
-        // only while that leaves most SMs idle
-        int BR = std::min(16, ntg);
-        while (BR > 4 && (long long)((ntg + BR - 1) / BR) * npc < 148) BR /= 2;
-        const size_t smem = (size_t)(BR + 4 + BR / 2) * p->Q * PC_ * sizeof(C) + (size_t)p->m2l_chunk * sizeof(R) +
-                            (size_t)2 * p->Q * p->Q * sizeof(R);
-        const dim3 grid((unsigned)((ntg + BR - 1) / BR), (unsigned)npc);
-        const R* tab = (const R*)p->m2l[lev];
-        with_pcd([&](auto pc) {
-            constexpr int PCv = decltype(pc)::value;
-            dispatch<2, 4, 8, 16>(BR, [&](auto br) {
-                constexpr int BRv = decltype(br)::value;
-                k_down<R, BRv, PCv><<<grid, PCv * p->Q, smem, s>>>(src, src_base, src_mod, parent, par_base, outp, tgt_base,
-                                                                   ntg, tab, p->m2l_chunk, (const R*)p->m2m, p->P, p->Q);
-            });
-        });
-        LAUNCH_CHECK();
         return FMMFFT_SUCCESS;
     }
 
@@ -1003,8 +1077,16 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
         cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
         const size_t scratch = ((size_t)Q << L) * p->esz;
         p->tree_p = (G == 1) && ((long long)Q << L) <= 8LL * threads && tree_p_smem(p, threads) + scratch <= (size_t)optin;
-        if (const char* e = getenv("FMMFFT_TREE")) p->tree_p = p->tree_p && e[0] == 'p';
+        if (const char* e = getenv("FMMFFT_TREE")) {
+            p->tree_p = p->tree_p && (e[0] == 'p' || e[0] == 'f');
+            p->tree_phased = e[0] == 'p';
+        }
     }
+    // tensor-core S2T: correct (parity-tested) but not yet faster end to end than the FFMA2 SIMT
+    // kernel on this workload, so opt-in: FMMFFT_S2T=tc
+    p->s2t_tc = false;
+    if (const char* e = getenv("FMMFFT_S2T"))
+        p->s2t_tc = e[0] == 't' && precision == FMMFFT_C64 && M_L == 64 && (p->nb % S2TC_BOXES) == 0;
     const char* g_env = getenv("FMMFFT_NO_GRAPH");
     p->use_graph = !(g_env && g_env[0] == '1');
     plan_radices(p);
@@ -1028,6 +1110,7 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
         if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&p->side, cudaStreamNonBlocking);
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->fork, cudaEventDisableTiming);
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->join, cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->fork2, cudaEventDisableTiming);
         if (e == cudaSuccess && (flags & FMMFFT_FLAG_PROFILE)) {
             e = cudaEventCreate(&p->ev_s2t[0]);
             if (e == cudaSuccess) e = cudaEventCreate(&p->ev_s2t[1]);

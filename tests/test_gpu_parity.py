@@ -211,3 +211,27 @@ def test_full_size_sampled(F, N, P, B, Q, prec, G):
     ny = np.sum(np.abs(y.astype(np.complex128)) ** 2)
     nx = np.sum(np.abs(x.astype(np.complex128)) ** 2)
     assert abs(ny / (N * nx) - 1) < 1e-5
+
+
+# ------------------------------------------------------------------ alternative kernel paths
+@pytest.mark.parametrize("env", [
+    {"FMMFFT_S2T": "tc"},        # S2T on tcgen05 (3xTF32, k_s2t_tc)
+    {"FMMFFT_TREE": "f"},        # far field fused in one per-FMM kernel (k_tree_pq)
+    {"FMMFFT_TREE": "w"},        # far field as wide per-level kernels (k_up, k_base, k_tree_down)
+    {"FMMFFT_NO_GRAPH": "1"},    # eager launches instead of a CUDA graph
+])
+@pytest.mark.parametrize("N,P,B,Q,G", [(1 << 20, 64, 2, 16, 1), (1 << 20, 64, 3, 16, 4)])
+def test_alternative_paths(F, monkeypatch, env, N, P, B, Q, G):
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)                   # read at plan creation
+    prec = "c64"
+    plan, x, y = run(F, N, P, B, Q, prec, 64, G=G, virtual=G > 1)
+    assert rel(y, O.fft_radix2(x)) < TOL_E2E[prec]
+    if G == 1:
+        L = O.tree_levels(N, P, 64)
+        st = O.fmm_stages(x.astype(np.complex128).reshape(2 ** L, 64, P), N, P, B, Q)
+        Tn = plan.debug_buffer("T_near").cpu().numpy().reshape(2 ** L, 64, P)
+        assert rel(Tn, st["T_near"]) < TOL_STAGE[prec]
+        assert np.array_equal(Tn[:, :, 0], x.reshape(2 ** L, 64, P)[:, :, 0])
+        LL = plan.debug_buffer("L", L).cpu().numpy().reshape(2 ** L, Q, P)
+        assert rel(LL[:, :, 1:], st["L"][L]) < TOL_STAGE[prec]
