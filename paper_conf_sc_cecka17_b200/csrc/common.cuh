@@ -75,4 +75,10 @@ template <int N> __device__ __forceinline__ void cp_async_wait_group() {
     asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory");
 }
 
+// Programmatic dependent launch: let the next kernel in the stream start scheduling its CTAs
+// (call early), and wait until the previous kernel's results are complete and visible (call
+// before the first read of them and before any global write).
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;\n" ::: "memory"); }
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;\n" ::: "memory"); }
+
 }  // namespace fmmfft

@@ -29,6 +29,7 @@
 #include <mutex>
 #include <string>
 #include <type_traits>
+#include <utility>
 #include <vector>
 
 #include "../../include/fmmfft.h"
@@ -76,6 +77,45 @@ static bool dispatch(int v, F&& f) {
     bool hit = false;
     ((v == Vs ? (f(std::integral_constant<int, Vs>{}), hit = true) : false), ...);
     return hit;
+}
+
+// Launch with programmatic dependent launch allowed: the kernel's CTAs may be scheduled while
+// its stream predecessor drains (each kernel triggers griddepcontrol.launch_dependents at its start
+// and waits in griddepcontrol.wait before touching the predecessor's results).
+static bool g_pdl = [] {
+    // Opt-in: measured on cfg2 (bench20) PDL cost 20 us/step (863 vs 1043 GFLOP/s) -- early
+    // dependent CTAs park in griddepcontrol.wait on SMs the side-stream S2T needs.
+    const char* e = getenv("FMMFFT_PDL");
+    return e && e[0] == '1';
+}();
+
+template <typename... KArgs, typename... Args>
+static cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args&&... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = g_pdl ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
+
+// Plain stream-ordered launch (for kernels whose CTAs fill an SM: launched early they would sit in
+// griddepcontrol.wait holding the SMs their predecessor and the side stream need).
+template <typename... KArgs, typename... Args>
+static cudaError_t launch_plain(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args&&... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cfg.attrs = nullptr;
+    cfg.numAttrs = 0;
+    return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
 }
 
 // ------------------------------------------------------------------ communicator
@@ -142,6 +182,7 @@ struct fmmfft_plan_s {
     int s2t_chunk = 0, m2l_chunk = 0, m2lB_chunk = 0;   // table chunk strides (elements)
     // device tables
     void* s2m = nullptr;
+    void* s2mT = nullptr;            // S2M^T [M_L][Qp], Qp = Q rounded up to 4 (k_s2m)
     void* m2m = nullptr;
     void* s2t = nullptr;
     void* rho = nullptr;
@@ -205,6 +246,13 @@ static fmmfft_status_t build_tables(fmmfft_plan_s* p) {
     for (int q = 0; q < Q; ++q)
         for (int m = 0; m < M_L; ++m) s2m[(size_t)q * M_L + m] = lagr(z, q, -1.0 + (2.0 * m + 1.0) / M_L);
     if ((st = upload<R>(p, &p->s2m, s2m))) return st;
+    {
+        const int Qp = (Q + 3) / 4 * 4;
+        std::vector<double> s2mT((size_t)M_L * Qp, 0.0);
+        for (int q = 0; q < Q; ++q)
+            for (int m = 0; m < M_L; ++m) s2mT[(size_t)m * Qp + q] = s2m[(size_t)q * M_L + m];
+        if ((st = upload<R>(p, &p->s2mT, s2mT))) return st;
+    }
     // M2M = [M2M^- M2M^+], M2M^{-+}_{qk} = l_q((z_k -+ 1)/2); L2L = M2M^T
     std::vector<double> m2m((size_t)Q * 2 * Q);
     for (int q = 0; q < Q; ++q)
@@ -499,24 +547,24 @@ struct Exec {
     // post_pfft), so the far field and the near field run concurrently
     fmmfft_status_t near_up() {
         fmmfft_status_t st;
-        // fork: the side stream starts after the S halo is in place
-        CUDA_TRY(cudaEventRecord(p->fork, s));
-        CUDA_TRY(cudaStreamWaitEvent(p->side, p->fork, 0));
         const int PCs = std::min(p->P, sizeof(R) == 4 ? 32 : 16);
         for (RankBufs& rb : p->ranks) {
             const C* S = in[p->virt ? rb.g : 0];
             const int Qp = (p->Q + 3) / 4 * 4;
-            const size_t smem = (size_t)p->M_L * PCs * sizeof(C) + (size_t)Qp * p->M_L * sizeof(R);
-            const dim3 grid((unsigned)p->nb, (unsigned)(p->P / PCs));
+            const int nbx = p->nb >= 2 ? 2 : 1;                // boxes per CTA (k_s2m NBX = 2; nb is even or 1)
+            const size_t smem = (size_t)2 * p->M_L * PCs * sizeof(C) + (size_t)Qp * p->M_L * sizeof(R);
+            const dim3 grid((unsigned)(p->nb / nbx), (unsigned)(p->P / PCs));
             dispatch<2, 4, 8, 16, 32>(PCs, [&](auto pc) {
                 constexpr int PCv = decltype(pc)::value;
                 if constexpr (!(sizeof(R) == 8 && PCv > 16))
-                    k_s2m<R, PCv><<<grid, PCv * (Qp / 4), smem, s>>>(S, interior(rb.Mpad[p->L]), (const R*)p->s2m, p->P,
-                                                                     p->M_L, p->Q, (C*)rb.Sp, p->nb);
+                    launch_pdl(k_s2m<R, PCv>, grid, PCv * (Qp / 4) * nbx, smem, s, S, interior(rb.Mpad[p->L]), (const R*)p->s2mT, p->P,
+                                                                           p->M_L, p->Q, (C*)rb.Sp, p->nb, nbx);
             });
             LAUNCH_CHECK();
         }
-        // S2T on the side stream
+        // fork after S2M (so S2M runs alone): S2T on the side stream
+        CUDA_TRY(cudaEventRecord(p->fork, s));
+        CUDA_TRY(cudaStreamWaitEvent(p->side, p->fork, 0));
         if ((st = mark_on(p->ev_s2t[0], p->side))) return st;
         if constexpr (sizeof(R) == 4) {
             if (p->s2t_tc) {                                   // tensor cores (tcgen05, 3xTF32)
@@ -529,7 +577,7 @@ struct Exec {
                     const C* hl = p->G == 1 ? S + (size_t)(p->nb - 1) * box : (const C*)rb.haloL;
                     const C* hr = p->G == 1 ? S : (const C*)rb.haloR;
                     const dim3 grid((unsigned)(p->nb / S2TC_BOXES), (unsigned)p->P);
-                    k_s2t_tc<<<grid, 256, s2tc_smem_bytes(), p->side>>>((const C*)rb.Sp, S, hl, hr, (C*)rb.Tn,
+                    launch_pdl(k_s2t_tc, grid, 256, s2tc_smem_bytes(), p->side, (const C*)rb.Sp, S, hl, hr, (C*)rb.Tn,
                                                                          (const float*)p->toep, p->P, p->nb, p->G);
                     LAUNCH_CHECK();
                 }
@@ -555,7 +603,7 @@ struct Exec {
                 constexpr int PCv = decltype(pc)::value;
                 if constexpr (sizeof(R) == 8 && PCv > 16) return;
                 else
-                    k_near_up<R, IB, PCv><<<grid, threads, smem, p->side>>>(S, hl, hr, (C*)rb.Tn, nullptr,
+                    launch_pdl(k_near_up<R, IB, PCv>, grid, threads, smem, p->side, S, hl, hr, (C*)rb.Tn, nullptr,
                                                                             (const R*)p->s2t, p->s2t_chunk, (const R*)p->s2m,
                                                                             p->P, p->M_L, p->Q, p->nb, bpc);
             };
@@ -590,7 +638,7 @@ struct Exec {
             const dim3 grid((unsigned)(nbc >> h), (unsigned)(p->P / PC_));
             with_pcd([&](auto pc) {
                 constexpr int PCv = decltype(pc)::value;
-                k_up<R, PCv><<<grid, PCv * p->Q, smem, s>>>(src, uo, h, (const R*)p->m2m, p->P, p->Q);
+                launch_pdl(k_up<R, PCv>, grid, PCv * p->Q, smem, s, src, uo, h, (const R*)p->m2m, p->P, p->Q);
             });
             LAUNCH_CHECK();
             src = (const C*)outs(cur - h);
@@ -620,8 +668,8 @@ struct Exec {
                     // (1) M2M + M2L-B + REDUCE per FMM, (2) all levels' M2L in one wide launch,
                     // (3) the L2L chain per FMM
                     const size_t smem1 = tree_p_smem(p, 512);
-                    if (p->Q == 16) k_tree_pq<16, 512, 8, false><<<p->P - 1, 512, smem1, s>>>(a, (const float*)p->m2m, p->P, tabB);
-                    else            k_tree_pq<8, 512, 8, false><<<p->P - 1, 512, smem1, s>>>(a, (const float*)p->m2m, p->P, tabB);
+                    if (p->Q == 16) launch_pdl(k_tree_pq<16, 512, 8, false>, p->P - 1, 512, smem1, s, a, (const float*)p->m2m, p->P, tabB);
+                    else            launch_pdl(k_tree_pq<8, 512, 8, false>, p->P - 1, 512, smem1, s, a, (const float*)p->m2m, p->P, tabB);
                     LAUNCH_CHECK();
                     if (p->L > p->B) {
                         M2LFlat f{};
@@ -643,20 +691,20 @@ struct Exec {
                         const dim3 grid((unsigned)tiles, (unsigned)(p->P / PC_));
                         with_pcd([&](auto pc) {
                             constexpr int PCv = decltype(pc)::value;
-                            k_m2l_flat<R, BR, PCv><<<grid, PCv * p->Q, smem2, s>>>(f, p->m2l_chunk, (const R*)p->m2m, p->P, p->Q);
+                            launch_pdl(k_m2l_flat<R, BR, PCv>, grid, PCv * p->Q, smem2, s, f, p->m2l_chunk, (const R*)p->m2m, p->P, p->Q);
                         });
                         LAUNCH_CHECK();
                         const size_t smem3 = (((size_t)2 << p->L) - ((size_t)1 << p->B)) * p->Q * sizeof(C) + (size_t)2 * p->Q * p->Q * sizeof(R);
-                        if (p->Q == 16) k_tree_dn<16, 512><<<p->P - 1, 512, smem3, s>>>(a, (const float*)p->m2m, p->P);
-                        else            k_tree_dn<8, 512><<<p->P - 1, 512, smem3, s>>>(a, (const float*)p->m2m, p->P);
+                        if (p->Q == 16) launch_pdl(k_tree_dn<16, 512>, p->P - 1, 512, smem3, s, a, (const float*)p->m2m, p->P);
+                        else            launch_pdl(k_tree_dn<8, 512>, p->P - 1, 512, smem3, s, a, (const float*)p->m2m, p->P);
                         LAUNCH_CHECK();
                     }
                     continue;
                 }
                 if ((p->Q == 16 || p->Q == 8) && (1LL << p->L) <= 8LL * ngrp) {
                     const size_t smem = tree_p_smem(p, 512) + ((size_t)p->Q << p->L) * sizeof(C);   // + scratch
-                    if (p->Q == 16) k_tree_pq<16, 512, 8><<<p->P - 1, 512, smem, s>>>(a, (const float*)p->m2m, p->P, tabB);
-                    else            k_tree_pq<8, 512, 8><<<p->P - 1, 512, smem, s>>>(a, (const float*)p->m2m, p->P, tabB);
+                    if (p->Q == 16) launch_plain(k_tree_pq<16, 512, 8>, p->P - 1, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
+                    else            launch_plain(k_tree_pq<8, 512, 8>, p->P - 1, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
                     LAUNCH_CHECK();
                     continue;
                 }
@@ -666,7 +714,7 @@ struct Exec {
             const size_t smem = tree_p_smem(p, threads);
             dispatch<1, 2, 4, 8>(maxo <= 1 ? 1 : maxo <= 2 ? 2 : maxo <= 4 ? 4 : 8, [&](auto mo) {
                 constexpr int MO = decltype(mo)::value;
-                k_tree_p<R, MO><<<p->P - 1, threads, smem, s>>>(a, (const R*)p->m2m, p->P, p->Q, tabB);
+                launch_plain(k_tree_p<R, MO>, p->P - 1, threads, smem, s, a, (const R*)p->m2m, p->P, p->Q, tabB);
             });
             LAUNCH_CHECK();
         }
@@ -734,7 +782,7 @@ struct Exec {
                 constexpr int PCv = decltype(pc)::value;
                 dispatch<4, 8, 16, 32>(NTr, [&](auto ntv) {
                     constexpr int NTv = decltype(ntv)::value;
-                    k_base<R, NTv, PCv><<<p->P / PCv, PCv * p->Q, smem, s>>>((const C*)rb.Mfull[p->B], outp, (C*)rb.r,
+                    launch_pdl(k_base<R, NTv, PCv>, p->P / PCv, PCv * p->Q, smem, s, (const C*)rb.Mfull[p->B], outp, (C*)rb.r,
                                                                            (int)tgt_base, ntg, (const R*)p->m2lB,
                                                                            p->m2lB_chunk, nbB, p->P, p->Q);
                 });
@@ -744,10 +792,10 @@ struct Exec {
         }
         const long long total = (long long)ntg * QP();
         const int blocks = (int)std::min<long long>((total + 255) / 256, 148LL * 16);
-        k_base_generic<R><<<blocks, 256, 0, s>>>((const C*)rb.Mfull[p->B], outp, tgt_base, ntg, (const R*)p->m2lB,
+        launch_pdl(k_base_generic<R>, blocks, 256, 0, s, (const C*)rb.Mfull[p->B], outp, tgt_base, ntg, (const R*)p->m2lB,
                                                   p->m2lB_chunk, PC_, nbB, p->P, p->Q);
         LAUNCH_CHECK();
-        k_reduce<R><<<(p->P + 127) / 128, 128, 0, s>>>((C*)rb.Mfull[p->B], (C*)rb.r, p->P, p->Q, nbB);
+        launch_pdl(k_reduce<R>, (p->P + 127) / 128, 128, 0, s, (C*)rb.Mfull[p->B], (C*)rb.r, p->P, p->Q, nbB);
         LAUNCH_CHECK();
         return FMMFFT_SUCCESS;
     }
@@ -818,7 +866,7 @@ struct Exec {
                 constexpr int PCv = decltype(pc)::value;
                 dispatch<1, 2, 4, 8, 16>(NR, [&](auto nr) {
                     constexpr int NRv = decltype(nr)::value;
-                    k_tree_down<R, PCv, NRv><<<grid, PCv * p->Q, smem, s>>>(a, (const R*)p->m2m, p->P, p->Q,
+                    launch_pdl(k_tree_down<R, PCv, NRv>, grid, PCv * p->Q, smem, s, a, (const R*)p->m2m, p->P, p->Q,
                                                                             p->m2l_chunk, db);
                 });
             });
@@ -838,7 +886,7 @@ struct Exec {
         for (RankBufs& rb : p->ranks) {
             dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 11>(ilog2(p->P), [&](auto lp) {
                 constexpr int LP = decltype(lp)::value;
-                k_post_pfft<R, LP><<<blocks, threads, smem, s>>>((const C*)rb.Tn, (const C*)rb.Lloc[p->L], (const C*)rb.r,
+                launch_pdl(k_post_pfft<R, LP>, blocks, threads, smem, s, (const C*)rb.Tn, (const C*)rb.Lloc[p->L], (const C*)rb.r,
                                                                 (const C*)p->rho, (const R*)p->s2m, (C*)rb.W,
                                                                 ilog2(p->M_L), p->Q, ilog2(MS), (int)p->Mg, stage_L);
             });
@@ -895,7 +943,7 @@ struct Exec {
                 const dim3 grid((unsigned)(nj / c), (unsigned)rows);
                 dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10>(lR, [&](auto lr) {
                     constexpr int LR = decltype(lr)::value;
-                    k_fft_pass<R, LR><<<grid, threads, smem, s>>>(src, o, lM, lNs, ilog2(c), in_row, lblk, blk_stride);
+                    launch_pdl(k_fft_pass<R, LR>, grid, threads, smem, s, src, o, lM, lNs, ilog2(c), in_row, lblk, blk_stride);
                 });
                 LAUNCH_CHECK();
                 src = o;
@@ -1106,8 +1154,12 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
         }
     }
     if (!st) {
-        cudaError_t e = cudaStreamCreateWithFlags(&p->cap_stream, cudaStreamNonBlocking);
-        if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&p->side, cudaStreamNonBlocking);
+        // the far field (main stream) is the critical path: it gets the higher priority, the near
+        // field on the side stream fills the SMs it leaves idle
+        int lo = 0, hi = 0;
+        cudaDeviceGetStreamPriorityRange(&lo, &hi);
+        cudaError_t e = cudaStreamCreateWithPriority(&p->cap_stream, cudaStreamNonBlocking, hi);
+        if (e == cudaSuccess) e = cudaStreamCreateWithPriority(&p->side, cudaStreamNonBlocking, lo);
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->fork, cudaEventDisableTiming);
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->join, cudaEventDisableTiming);
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->fork2, cudaEventDisableTiming);

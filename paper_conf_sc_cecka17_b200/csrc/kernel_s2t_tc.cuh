@@ -38,6 +38,8 @@ __host__ __device__ constexpr size_t s2tc_smem_bytes() {
 __global__ void __launch_bounds__(256, 2)
 k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ S, const float2* __restrict__ haloL,
          const float2* __restrict__ haloR, float2* __restrict__ Tn, const float* __restrict__ toep, int P, int nb, int G) {
+    pdl_trigger();
+    pdl_wait();
     extern __shared__ __align__(1024) unsigned char smem_tc[];
     float2* Scol = reinterpret_cast<float2*>(smem_tc);                           // [66][64]
     unsigned char* Abase = smem_tc + S2TC_SCOL_BYTES;                            // 2 x (hi, lo)

@@ -140,6 +140,7 @@ __global__ void __launch_bounds__(sizeof(R) == 4 ? 1024 : 512)
 k_post_pfft(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2<R>* __restrict__ r,
             const C2<R>* __restrict__ rho, const R* __restrict__ s2m, C2<R>* __restrict__ W,
             int lML, int Q, int lMS, int Mg, int stage_L) {
+    pdl_trigger();
     using C = C2<R>;
     constexpr int P = 1 << LP, LD = P + 1;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -152,13 +153,14 @@ k_post_pfft(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2
     const int lnsub = lML - lMS;
     const int b = blockIdx.x >> lnsub, m0 = (blockIdx.x & ((1 << lnsub) - 1)) << lMS;
 
+    for (int idx = tid; idx < Q * MS; idx += nthr) cp_async_elem(s2m_sm + idx, s2m + (idx >> lMS) * M_L + m0 + (idx & (MS - 1)));
+    fill_twiddles<R>(tw, LP);
+    pdl_wait();                                                   // T_near / L^L / r from the FMM stages
     const C* src = Tn + (((size_t)b << lML) + m0) * P;
     for (int idx = tid; idx < (MS << LP); idx += nthr) cp_async_elem(tile + (idx >> LP) * LD + (idx & (P - 1)), src + idx);
     const C* Lb = LL + (size_t)b * Q * P;
     if (stage_L)
         for (int idx = tid; idx < Q * P; idx += nthr) cp_async_elem(Lsm + idx, Lb + idx);
-    for (int idx = tid; idx < Q * MS; idx += nthr) cp_async_elem(s2m_sm + idx, s2m + (idx >> lMS) * M_L + m0 + (idx & (MS - 1)));
-    fill_twiddles<R>(tw, LP);
     cp_async_wait_all();
     __syncthreads();
 
@@ -212,6 +214,7 @@ template <typename R, int LR>
 __global__ void __launch_bounds__(sizeof(R) == 4 ? 1024 : 512)
 k_fft_pass(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, int lM, int lNs, int lc,
            int in_row, int lblk, int blk_stride) {
+    pdl_trigger();
     using C = C2<R>;
     constexpr int Rp = 1 << LR, LD = Rp + 1;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -228,6 +231,8 @@ k_fft_pass(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, int lM, int lN
     const C* xin = in + row * (size_t)in_row;
     const int total = c << LR;
 
+    fill_twiddles<R>(tw, LR);                                     // independent of the predecessor
+    pdl_wait();
     // 8 elements per thread: all loads issued before any is used
     C v[8];
 #pragma unroll
@@ -239,7 +244,6 @@ k_fft_pass(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, int lM, int lN
             v[u] = ldg_c(xin + (size_t)(m >> lblk) * blk_stride + (m & bmask));
         }
     }
-    fill_twiddles<R>(tw, LR);
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
         const int idx = tid + u * nthr;
