@@ -109,14 +109,36 @@ def load_peaks():
         return {}
 
 
-def load_traffic(workload: str, G: int):
-    """Per-launch DRAM bytes of near_up from the committed ncu --set full summary, if any."""
+def load_traffic(workload: str, G: int, kernel: str):
+    """Per-launch DRAM bytes (dram__bytes_read.sum + dram__bytes_write.sum) of one kernel from the
+    committed `ncu --set full` summary (profiles/ncu_traffic.json), if it was captured."""
     try:
         d = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
-        e = d.get(f"{workload}_G{G}")
-        return e and e.get("near_up_dram_bytes")
+        e = d.get(f"{workload}_G{G}", {}).get(kernel)
+        return e and e.get("dram_bytes")
     except Exception:
         return None
+
+
+def stage_rooflines(N, P, B, Q, M_L, G, L, prec, tree_fused):
+    """Algorithmic work per launch of each kernel stage, restated from PAPER.md §5.1:
+    complex x real multiply-adds cost 2C = 4 real flops; the FFT stages are HBM-bound and move
+    their input and output once. Returns {stage: (kernel, bound, amount)}."""
+    C, nb = 2, 2 ** L / G
+    fmm = P - 1
+    esz = 8 if prec == "c64" else 16
+    up = sum(2 ** l for l in range(B, L)) / G                      # parents formed by M2M
+    dn = sum(2 ** l for l in range(B + 1, L + 1)) / G              # targets of M2L / L2L
+    tree = 2 * C * fmm * Q * Q * (2 * up + 3 * dn + dn) + 2 * C * fmm * Q * Q * 2 ** B * (2 ** B - 3) / G
+    out = {
+        "s2m": ("k_s2m", "alu", 2 * C * M_L * nb * fmm * Q),
+        "s2t": ("k_near_up", "alu", 6 * C * M_L * M_L * nb * fmm),
+        "post_pfft": ("k_post_pfft", "hbm", (N // G) * esz * 2 + nb * Q * P * esz),
+        "mfft": ("k_fft_pass / k_fft_row", "hbm", (N // G) * esz * 2),
+    }
+    if tree_fused:
+        out["top"] = ("k_tree_pq", "alu", tree)
+    return out
 
 
 # ------------------------------------------------------------------------------ CPU oracle legs
@@ -326,14 +348,29 @@ def run_fmmfft(args, rank, world, local_rank):
     if rank != 0:
         return
     peaks = load_peaks()
-    fl = s2t_flops(N, P, M_L, G)
-    t_near = stages.get("s2t", float("nan")) * 1e-3
     sm_max = peaks.get("sm_max_mhz", 1965.0)
     if prec == "c64":
-        peak = 148 * 128 * 2 * sm_max * 1e6 / 1e12            # FP32 FMA lanes x 2 flops x max clock
+        alu_peak = 148 * 128 * 2 * sm_max * 1e6 / 1e12        # FP32 FMA lanes x 2 flops x max clock
     else:
-        peak = 148 * 64 * 2 * sm_max * 1e6 / 1e12             # FP64 FMA lanes (half rate)
-    achieved = fl / t_near / 1e12
+        alu_peak = 148 * 64 * 2 * sm_max * 1e6 / 1e12         # FP64 FMA lanes (half rate)
+    hbm_peak = peaks.get("hbm_gbs", 6454.3)
+    rl = {}
+    for st_name, (kname, bound, amount) in stage_rooflines(N, P, B, Q, M_L, G, info["L"], prec,
+                                                           bool(info["variant"] & 1)).items():
+        t = stages.get(st_name)
+        if not t or t != t:
+            continue
+        if bound == "alu":
+            ach, pk, unit = amount / (t * 1e-3) / 1e12, alu_peak, "TFLOP/s"
+        else:
+            ach, pk, unit = amount / (t * 1e-3) / 1e9, hbm_peak, "GB/s"
+        rl[st_name] = {"kernel": kname, "bound": bound, "achieved": ach, "peak": pk, "unit": unit, "frac": ach / pk,
+                       "traffic": load_traffic(workload, G, kname.split(" ")[0]), "avg_launch_ms": t,
+                       ("algorithmic_flops_per_launch" if bound == "alu" else "algorithmic_bytes_per_launch"): amount}
+    dom = max(rl, key=lambda k: rl[k]["avg_launch_ms"])
+    roof = dict(rl[dom], stage=dom,
+                peak_basis=(f"148 SMs x {'128 FP32' if prec == 'c64' else '64 FP64'} FMA/clk x 2 x {sm_max} MHz (guide unit counts)"
+                            if rl[dom]["bound"] == "alu" else "MEASURED_PEAKS.json HBM copy bandwidth"))
     clocks = sampler.summary()
     line = {
         "metric": "1D C2C FFT GFLOP/s (5N log2N/t)", "value": value, "unit": "GFLOP/s", "n_gpus": world,
@@ -343,10 +380,8 @@ def run_fmmfft(args, rank, world, local_rank):
         "config": {"workload": workload, "desc": desc, "N": N, "P": P, "G": G, "B": B, "Q": Q, "M_L": M_L,
                    "L": info["L"], "precision": prec, "l2": "flushed (256 MiB write between steps, outside events)",
                    "parseval_rel_dev": parseval},
-        "roofline": {"kernel": "k_near_up (S2T, side stream, concurrent with the far field)", "bound": "alu", "achieved": achieved, "peak": peak,
-                     "unit": "TFLOP/s", "frac": achieved / peak, "traffic": load_traffic(workload, G),
-                     "algorithmic_flops_per_launch": fl, "avg_launch_ms": t_near * 1e3,
-                     "peak_basis": f"148 SMs x {'128 FP32' if prec == 'c64' else '64 FP64'} FMA/clk x 2 x {sm_max} MHz"},
+        "roofline": roof,
+        "stages_roofline": rl,
         "stages_ms": stages,
         "e2e": {"value": flops_fft(N) / (e2e_ms * 1e-3) / 1e9, "unit": "GFLOP/s",
                 "h2d_bytes_per_step": (N // G) * esz, "d2h_bytes_per_step": (N // G) * esz, "ms_per_step": e2e_ms},

@@ -115,7 +115,12 @@ typedef struct {
     int n_stages;           /* entries reported by fmmfft_stage_times               */
     size_t workspace_bytes; /* device bytes owned by the plan (all virtual ranks)   */
     int kernels_per_execute;/* kernels this library launched in the last execute (0 before) */
+    unsigned variant;       /* kernel variants the plan chose: FMMFFT_VARIANT_* bits below  */
 } fmmfft_info_t;
+
+#define FMMFFT_VARIANT_TREE_FUSED 1u  /* far field as one per-FMM kernel (G = 1, tree fits smem) */
+#define FMMFFT_VARIANT_S2T_TC     2u  /* near field on tcgen05 tensor cores (3xTF32)             */
+#define FMMFFT_VARIANT_ROW_FFT1   4u  /* M-point FFTs as one single-pass kernel per row        */
 
 FMMFFT_API fmmfft_status_t fmmfft_get_info(fmmfft_plan_t plan, fmmfft_info_t* info);
 

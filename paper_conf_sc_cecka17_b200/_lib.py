@@ -27,7 +27,8 @@ class Info(ctypes.Structure):
     _fields_ = [("N", ctypes.c_longlong), ("P", ctypes.c_int), ("G", ctypes.c_int), ("B", ctypes.c_int),
                 ("Q", ctypes.c_int), ("M_L", ctypes.c_int), ("L", ctypes.c_int), ("precision", ctypes.c_int),
                 ("M", ctypes.c_longlong), ("level_gather", ctypes.c_int), ("n_stages", ctypes.c_int),
-                ("workspace_bytes", ctypes.c_size_t), ("kernels_per_execute", ctypes.c_int)]
+                ("workspace_bytes", ctypes.c_size_t), ("kernels_per_execute", ctypes.c_int),
+                ("variant", ctypes.c_uint)]
 
 
 class FmmfftError(RuntimeError):
