@@ -193,6 +193,8 @@ struct fmmfft_plan_s {
     bool tree_phased = false;        // ... as up / all-levels M2L / L2L-chain launches (FMMFFT_TREE=p) (k_tree_pq<.., false>, k_m2l_flat, k_tree_dn)
     bool s2t_tc = false;             // S2T on tcgen05 (k_s2t_tc): complex64, M_L = 64, nb % 64 == 0
     void* toep = nullptr;            // its Toeplitz hi/lo operand table
+    bool row_fft1 = false;           // M-point FFTs in one pass per row (k_fft_row), M fits smem
+    void* twM = nullptr;             // its twiddles w_M^u, u < M/16
     std::vector<fmmfft::RankBufs> ranks;
     std::vector<int> radices;        // M-FFT passes
     size_t ws_bytes = 0;
@@ -342,10 +344,20 @@ static fmmfft_status_t build_tables(fmmfft_plan_s* p) {
         rho[2 * pp] = pp ? std::cos(M_PI * pp / P) * sn : 1.0;
         rho[2 * pp + 1] = pp ? -std::sin(M_PI * pp / P) * sn : 0.0;
     }
-    return upload<R>(p, &p->rho, rho);
+    if ((st = upload<R>(p, &p->rho, rho))) return st;
+    if (p->row_fft1) {                                   // w_M^u = exp(-2 pi i u / M), u < M/16
+        std::vector<double> tw(2 * (p->M / 16));
+        for (long long u = 0; u < p->M / 16; ++u) {
+            tw[2 * u] = std::cos(2 * M_PI * (double)u / (double)p->M);
+            tw[2 * u + 1] = -std::sin(2 * M_PI * (double)u / (double)p->M);
+        }
+        if ((st = upload<R>(p, &p->twM, tw))) return st;
+    }
+    return FMMFFT_SUCCESS;
 }
 
 static constexpr int kTileF = 8192, kTileD = 4096;   // shared FFT tile (elements)
+template <typename R> static constexpr int kRowFftMax = sizeof(R) == 4 ? 14 : 13;   // k_fft_row: whole row in smem
 
 static void plan_radices(fmmfft_plan_s* p) {
     const int maxbits = p->prec == FMMFFT_C64 ? 10 : 9;
@@ -464,6 +476,10 @@ static fmmfft_status_t init_kernel_attrs() {
             dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 11>(lp, [&](auto v) { set((const void*)k_post_pfft<R, decltype(v)::value>); });
         for (int lr = 1; lr <= 10; ++lr)
             dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10>(lr, [&](auto v) { set((const void*)k_fft_pass<R, decltype(v)::value>); });
+        for (int ll = 8; ll <= kRowFftMax<R>; ++ll)
+            dispatch<8, 9, 10, 11, 12, 13, 14>(ll, [&](auto v) {
+                if constexpr (decltype(v)::value <= kRowFftMax<R>) set((const void*)k_fft_row<R, decltype(v)::value>);
+            });
     });
     CUDA_TRY(err);
     return FMMFFT_SUCCESS;
@@ -926,6 +942,19 @@ struct Exec {
         for (RankBufs& rb : p->ranks) {
             C* dst = out[p->virt ? rb.g : 0];
             const C* src = (const C*)(p->G > 1 ? rb.Rcv : rb.W);
+            if (p->row_fft1) {                   // one pass per row, the row in shared memory
+                int in_row = (int)p->M, lblk = lM, blk_stride = 0;
+                if (p->G > 1) { in_row = (int)p->Mg; lblk = ilog2(p->Mg); blk_stride = (int)((p->P / p->G) * p->Mg); }
+                const size_t smem = ((size_t)p->M + p->M / 16 + p->M / 16) * sizeof(C);
+                dispatch<8, 9, 10, 11, 12, 13, 14>(lM, [&](auto ll) {
+                    constexpr int LL = decltype(ll)::value;
+                    if constexpr (LL <= kRowFftMax<R>)
+                        launch_pdl(k_fft_row<R, LL>, (unsigned)rows, 1 << (LL - 4), smem, s, src, dst, (const C*)p->twM,
+                                   in_row, lblk, blk_stride);
+                });
+                LAUNCH_CHECK();
+                continue;
+            }
             int lNs = 0;
             for (int i = 0; i < n; ++i) {
                 const int Rp = p->radices[i], lR = ilog2(Rp);
@@ -1138,6 +1167,11 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
     const char* g_env = getenv("FMMFFT_NO_GRAPH");
     p->use_graph = !(g_env && g_env[0] == '1');
     plan_radices(p);
+    {
+        const int lM = ilog2(p->M);
+        const char* e = getenv("FMMFFT_ROWFFT");
+        p->row_fft1 = lM >= 8 && lM <= (precision == FMMFFT_C64 ? 14 : 13) && !(e && e[0] == '0');
+    }
     st = precision == FMMFFT_C64 ? build_tables<float>(p) : build_tables<double>(p);
     if (!st) {
         const int nr = virt ? G : 1;
@@ -1229,7 +1263,8 @@ fmmfft_status_t fmmfft_get_info(fmmfft_plan_t p, fmmfft_info_t* info) {
     info->N = p->N; info->P = p->P; info->G = p->G; info->B = p->B; info->Q = p->Q; info->M_L = p->M_L;
     info->L = p->L; info->precision = p->prec; info->M = p->M; info->level_gather = p->lg;
     info->n_stages = ST_COUNT + 1; info->workspace_bytes = p->ws_bytes; info->kernels_per_execute = p->kernels;
-    info->variant = (p->tree_p ? FMMFFT_VARIANT_TREE_FUSED : 0u) | (p->s2t_tc ? FMMFFT_VARIANT_S2T_TC : 0u);
+    info->variant = (p->tree_p ? FMMFFT_VARIANT_TREE_FUSED : 0u) | (p->s2t_tc ? FMMFFT_VARIANT_S2T_TC : 0u) |
+                    (p->row_fft1 ? FMMFFT_VARIANT_ROW_FFT1 : 0u);
     return FMMFFT_SUCCESS;
 }
 

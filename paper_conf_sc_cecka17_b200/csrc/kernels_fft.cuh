@@ -275,4 +275,136 @@ k_fft_pass(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, int lM, int lN
     }
 }
 
+// ---------------------------------------------------------------------------------------------
+// k_fft_row: the whole M-point FFT of one row in ONE pass (§3 step 4), for rows that fit
+// in shared memory (M = 2^LLEN <= 2^14 complex64 / 2^13 complex128). Stockham autosort with a
+// first stage of radix R0 = 2^(LLEN mod 4) (16 if that is 0) and radix-16 stages after it; a
+// thread owns 16 elements per stage (16/r butterflies), M/16 threads per row:
+//   stage (r, Ns): for j < M/r, k = j mod Ns:
+//     v_t = x[j + t M/r] w_{r Ns}^{k t},  v = DFT_r(v),  y[(j - k) r + k + t Ns] = v_t.
+// The first stage reads the row straight from global memory (the all-to-all receive layout as
+// in k_fft_pass), the last (r = 16, Ns = M/16, so k = j) stores y[j + t M/16] — natural order —
+// straight to global memory; in between, shared memory with one pad element per 16 (the
+// stride-4 / stride-r write patterns land on distinct banks). Twiddles: w_M^u for u < M/16 from
+// a host-computed (fp64) table; the powers w^t, t < 16, by a depth-4 product tree.
+// ---------------------------------------------------------------------------------------------
+template <typename C, typename Rr>
+__device__ __forceinline__ C cmul_k(C a, Rr re, Rr im) {         // a * (re + i im), constants
+    C r;
+    r.x = a.x * re - a.y * im;
+    r.y = a.x * im + a.y * re;
+    return r;
+}
+
+// X[k] = sum_n v[n] w_16^{nk}, natural order in and out: 4 x 4 with inner twiddles w_16^{n2 k1}
+template <typename C> __device__ __forceinline__ void dft16(C* v) {
+    using R = decltype(v[0].x);
+    const R c1 = (R)0.92387953251128675613, s1 = (R)0.38268343236508977173, h = (R)0.70710678118654752440;
+    C a[4][4];
+#pragma unroll
+    for (int n2 = 0; n2 < 4; ++n2) {
+        C t[4] = {v[n2], v[4 + n2], v[8 + n2], v[12 + n2]};
+        dft4(t);
+#pragma unroll
+        for (int k1 = 0; k1 < 4; ++k1) a[n2][k1] = t[k1];
+    }
+    // w16^1 = (c1,-s1), w16^2 = (h,-h), w16^3 = (s1,-c1), w16^4 = -i, w16^6 = (-h,-h), w16^9 = (-c1,s1)
+    a[1][1] = cmul_k(a[1][1], c1, -s1);
+    a[1][2] = cmul_k(a[1][2], h, -h);
+    a[1][3] = cmul_k(a[1][3], s1, -c1);
+    a[2][1] = cmul_k(a[2][1], h, -h);
+    a[2][2] = mul_mi(a[2][2]);
+    a[2][3] = cmul_k(a[2][3], -h, -h);
+    a[3][1] = cmul_k(a[3][1], s1, -c1);
+    a[3][2] = cmul_k(a[3][2], -h, -h);
+    a[3][3] = cmul_k(a[3][3], -c1, s1);
+#pragma unroll
+    for (int k1 = 0; k1 < 4; ++k1) {
+        C t[4] = {a[0][k1], a[1][k1], a[2][k1], a[3][k1]};
+        dft4(t);
+#pragma unroll
+        for (int k2 = 0; k2 < 4; ++k2) v[k1 + 4 * k2] = t[k2];
+    }
+}
+
+template <int E, typename C> __device__ __forceinline__ void dftR(C* v) {
+    if constexpr (E == 16) dft16(v);
+    else dftE<E>(v);
+}
+
+// v[t] *= w^t for t = 1 .. E-1 (w^t by a product tree of depth <= 4)
+template <int E, typename C> __device__ __forceinline__ void twiddle_powers(C* v, C w1) {
+    C w[E];
+    w[1] = w1;
+#pragma unroll
+    for (int t = 2; t < E; ++t) w[t] = (t & 1) ? cmul(w[t - 1], w1) : cmul(w[t / 2], w[t / 2]);
+#pragma unroll
+    for (int t = 1; t < E; ++t) v[t] = cmul(v[t], w[t]);
+}
+
+__device__ __forceinline__ constexpr int row_pad(int a) { return a + (a >> 4); }
+
+template <typename R, int LLEN>
+__global__ void __launch_bounds__(1 << (LLEN - 4))
+k_fft_row(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, const C2<R>* __restrict__ twM,
+          int in_row, int lblk, int blk_stride) {
+    using C = C2<R>;
+    constexpr int M = 1 << LLEN, NT = M >> 4;
+    constexpr int L0 = (LLEN & 3) ? (LLEN & 3) : 4, R0 = 1 << L0, NB0 = 16 / R0;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    C* x = reinterpret_cast<C*>(smem_raw);                        // [row_pad(M)]
+    C* tw = x + row_pad(M);                                       // [M/16]  w_M^u
+    const int tid = threadIdx.x;
+    for (int u = tid; u < NT; u += NT) cp_async_elem(tw + u, twM + u);
+    cp_async_commit();
+
+    // ---- stage 0: radix R0, Ns = 1, from global (no twiddles)
+    const C* xin = in + (size_t)blockIdx.x * in_row;
+    const int bmask = (1 << lblk) - 1;
+    C v[16];
+#pragma unroll
+    for (int b = 0; b < NB0; ++b) {
+        const int j = tid + b * NT;
+#pragma unroll
+        for (int t = 0; t < R0; ++t) {
+            const int m = j + t * (M / R0);
+            v[b * R0 + t] = ldg_c(xin + (size_t)(m >> lblk) * blk_stride + (m & bmask));
+        }
+    }
+#pragma unroll
+    for (int b = 0; b < NB0; ++b) dftR<R0>(v + b * R0);
+#pragma unroll
+    for (int b = 0; b < NB0; ++b) {
+        const int j = tid + b * NT;
+#pragma unroll
+        for (int t = 0; t < R0; ++t) x[row_pad(j * R0 + t)] = v[b * R0 + t];
+    }
+    cp_async_wait_all();
+    __syncthreads();
+
+    // ---- radix-16 stages, Ns = R0, 16 R0, ...; the last one (Ns = M/16) stores to global
+    auto stage = [&](auto lnsc) {
+        constexpr int LNS = decltype(lnsc)::value, NS = 1 << LNS;
+        const int j = tid, k = j & (NS - 1);
+#pragma unroll
+        for (int t = 0; t < 16; ++t) v[t] = x[row_pad(j + t * NT)];
+        twiddle_powers<16>(v, tw[k << (LLEN - 4 - LNS)]);
+        dft16(v);
+        if constexpr (LNS + 4 < LLEN) {
+            __syncthreads();
+#pragma unroll
+            for (int t = 0; t < 16; ++t) x[row_pad(((j - k) << 4) + k + t * NS)] = v[t];
+            __syncthreads();
+        } else {
+            C* y = out + ((size_t)blockIdx.x << LLEN);
+#pragma unroll
+            for (int t = 0; t < 16; ++t) y[j + t * NT] = v[t];
+        }
+    };
+    stage(std::integral_constant<int, L0>{});
+    if constexpr (L0 + 4 < LLEN) stage(std::integral_constant<int, L0 + 4>{});
+    if constexpr (L0 + 8 < LLEN) stage(std::integral_constant<int, L0 + 8>{});
+    static_assert(L0 + 12 >= LLEN, "k_fft_row: LLEN <= L0 + 12");
+}
+
 }  // namespace fmmfft

@@ -219,6 +219,7 @@ def test_full_size_sampled(F, N, P, B, Q, prec, G):
     {"FMMFFT_TREE": "f"},        # far field fused in one per-FMM kernel (k_tree_pq)
     {"FMMFFT_TREE": "w"},        # far field as wide per-level kernels (k_up, k_base, k_tree_down)
     {"FMMFFT_NO_GRAPH": "1"},    # eager launches instead of a CUDA graph
+    {"FMMFFT_ROWFFT": "0"},      # multi-pass M-point FFT (k_fft_pass) instead of k_fft_row
 ])
 @pytest.mark.parametrize("N,P,B,Q,G", [(1 << 20, 64, 2, 16, 1), (1 << 20, 64, 3, 16, 4)])
 def test_alternative_paths(F, monkeypatch, env, N, P, B, Q, G):
