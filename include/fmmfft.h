@@ -64,6 +64,10 @@ typedef enum {
                                    are then the FULL length-N vectors. For testing the
                                    partitioned algorithm on one GPU. */
 #define FMMFFT_FLAG_PROFILE 2u  /* record CUDA events around every stage (fmmfft_stage_times) */
+#define FMMFFT_FLAG_DEBUG 4u    /* keep every level's M^l / L^l in the buffers fmmfft_debug_buffer
+                                   returns. Without it the fused single-GPU far field
+                                   (FMMFFT_VARIANT_TREE_FUSED) keeps levels < L on chip only, and
+                                   those debug buffers hold stale data. */
 
 /* ---------------------------------------------------------------- communicator (G > 1)
  * One process per GPU. Rank 0 calls fmmfft_get_unique_id and broadcasts the 128 bytes (e.g.

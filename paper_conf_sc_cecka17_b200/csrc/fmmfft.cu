@@ -473,7 +473,12 @@ static fmmfft_status_t init_kernel_attrs() {
         set((const void*)k_tree_p<R, 4>);
         set((const void*)k_tree_p<R, 8>);
         for (int lp = 1; lp <= 11; ++lp)
-            dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 11>(lp, [&](auto v) { set((const void*)k_post_pfft<R, decltype(v)::value>); });
+            dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 11>(lp, [&](auto v) {
+                set((const void*)k_post_pfft<R, decltype(v)::value, 0>);
+                set((const void*)k_post_pfft<R, decltype(v)::value, 8>);
+                set((const void*)k_post_pfft<R, decltype(v)::value, 16>);
+                set((const void*)k_post_pfft<R, decltype(v)::value, 24>);
+            });
         for (int lr = 1; lr <= 10; ++lr)
             dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10>(lr, [&](auto v) { set((const void*)k_fft_pass<R, decltype(v)::value>); });
         for (int ll = 8; ll <= kRowFftMax<R>; ++ll)
@@ -676,6 +681,7 @@ struct Exec {
             a.r = rb.r;
             a.L = p->L;
             a.B = p->B;
+            a.dbg = (p->flags & FMMFFT_FLAG_DEBUG) ? 1 : 0;
             const int tabB = ((1 << p->B) - 3) * p->Q * p->Q;
             // complex64 with Q = 16 or 8 and <= 8 boxes per thread group: register-blocked kernel
             if constexpr (sizeof(R) == 4) {
@@ -718,7 +724,9 @@ struct Exec {
                     continue;
                 }
                 if ((p->Q == 16 || p->Q == 8) && (1LL << p->L) <= 8LL * ngrp) {
-                    const size_t smem = tree_p_smem(p, 512) + ((size_t)p->Q << p->L) * sizeof(C);   // + scratch
+                    // + L2L rows as float2 + the two alternating L^l buffers (2^L and 2^(L-1) boxes)
+                    const size_t smem = tree_p_smem(p, 512) + (size_t)p->Q * p->Q * 2 * sizeof(R) +
+                                        (((size_t)3 * p->Q) << (p->L - 1)) * sizeof(C);
                     if (p->Q == 16) launch_plain(k_tree_pq<16, 512, 8>, p->P - 1, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
                     else            launch_plain(k_tree_pq<8, 512, 8>, p->P - 1, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
                     LAUNCH_CHECK();
@@ -900,11 +908,14 @@ struct Exec {
         if (stage_L) smem += (size_t)p->Q * p->P * sizeof(C);
         const int blocks = p->nb * (p->M_L / MS);
         for (RankBufs& rb : p->ranks) {
+            const int qt = (p->Q == 8 || p->Q == 16 || p->Q == 24) ? p->Q : 0;
             dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 11>(ilog2(p->P), [&](auto lp) {
                 constexpr int LP = decltype(lp)::value;
-                launch_pdl(k_post_pfft<R, LP>, blocks, threads, smem, s, (const C*)rb.Tn, (const C*)rb.Lloc[p->L], (const C*)rb.r,
-                                                                (const C*)p->rho, (const R*)p->s2m, (C*)rb.W,
-                                                                ilog2(p->M_L), p->Q, ilog2(MS), (int)p->Mg, stage_L);
+                dispatch<0, 8, 16, 24>(qt, [&](auto qv) {
+                    launch_pdl(k_post_pfft<R, LP, decltype(qv)::value>, blocks, threads, smem, s, (const C*)rb.Tn,
+                               (const C*)rb.Lloc[p->L], (const C*)rb.r, (const C*)p->rho, (const R*)p->s2m, (C*)rb.W,
+                               ilog2(p->M_L), p->Q, ilog2(MS), (int)p->Mg, stage_L);
+                });
             });
             LAUNCH_CHECK();
         }
@@ -1152,7 +1163,7 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
         const int threads = precision == FMMFFT_C64 ? 1024 : 512;
         int optin = 0;
         cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-        const size_t scratch = ((size_t)Q << L) * p->esz;
+        const size_t scratch = (((size_t)3 * Q) << (L > 0 ? L - 1 : 0)) * p->esz + (size_t)2 * Q * Q * p->rsz;
         p->tree_p = (G == 1) && ((long long)Q << L) <= 8LL * threads && tree_p_smem(p, threads) + scratch <= (size_t)optin;
         if (const char* e = getenv("FMMFFT_TREE")) {
             p->tree_p = p->tree_p && (e[0] == 'p' || e[0] == 'f');

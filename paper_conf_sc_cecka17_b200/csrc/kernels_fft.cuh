@@ -135,59 +135,84 @@ __device__ __forceinline__ void fill_twiddles(C2<R>* tw, int llen) {
 // Mg = M/G (this rank's m range): element (k2, m_local) at W[k2 * Mg + m_local] — the
 // all-to-all send layout [destination r][k2 local][m local] with k2 = r P/G + k2 local.
 // ---------------------------------------------------------------------------------------------
-template <typename R, int LP>
+template <typename R, int LP, int QT>
 __global__ void __launch_bounds__(sizeof(R) == 4 ? 1024 : 512)
 k_post_pfft(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2<R>* __restrict__ r,
             const C2<R>* __restrict__ rho, const R* __restrict__ s2m, C2<R>* __restrict__ W,
-            int lML, int Q, int lMS, int Mg, int stage_L) {
+            int lML, int Qrt, int lMS, int Mg, int stage_L) {
     pdl_trigger();
     using C = C2<R>;
     constexpr int P = 1 << LP, LD = P + 1;
+    constexpr int MG = 8;                                         // m per thread in L2T + POST
     extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int Q = QT ? QT : Qrt;
     const int MS = 1 << lMS, M_L = 1 << lML;
     C* tile = reinterpret_cast<C*>(smem_raw);                    // [MS][P + 1]
     C* tw = tile + MS * LD;                                       // [P]
     C* Lsm = tw + P;                                              // [Q][P]   L^L of box b (if staged)
-    R* s2m_sm = reinterpret_cast<R*>(Lsm + (stage_L ? Q * P : 0)); // [Q][MS]
+    R* s2m_sm = reinterpret_cast<R*>(Lsm + (stage_L ? Q * P : 0)); // [Q][MS]  (16-byte aligned: MS % 8 == 0)
     const int tid = threadIdx.x, nthr = blockDim.x;
     const int lnsub = lML - lMS;
     const int b = blockIdx.x >> lnsub, m0 = (blockIdx.x & ((1 << lnsub) - 1)) << lMS;
 
-    for (int idx = tid; idx < Q * MS; idx += nthr) cp_async_elem(s2m_sm + idx, s2m + (idx >> lMS) * M_L + m0 + (idx & (MS - 1)));
+    // constants (independent of the FMM stages): L2T rows of this m sub-tile, twiddles
+    {
+        constexpr int V = 16 / sizeof(R);                         // R per 16-byte copy
+        const int nv = (Q * MS) / V, vpr = MS / V;
+        for (int idx = tid; idx < nv; idx += nthr) {
+            const int q = idx / vpr, c = idx - q * vpr;
+            cp_async<16>(s2m_sm + q * MS + c * V, s2m + (size_t)q * M_L + m0 + c * V);
+        }
+    }
     fill_twiddles<R>(tw, LP);
     pdl_wait();                                                   // T_near / L^L / r from the FMM stages
-    const C* src = Tn + (((size_t)b << lML) + m0) * P;
-    for (int idx = tid; idx < (MS << LP); idx += nthr) cp_async_elem(tile + (idx >> LP) * LD + (idx & (P - 1)), src + idx);
-    const C* Lb = LL + (size_t)b * Q * P;
-    if (stage_L)
-        for (int idx = tid; idx < Q * P; idx += nthr) cp_async_elem(Lsm + idx, Lb + idx);
+    {
+        // T_near rows [m][p] (contiguous P per m) -> tile rows (stride P + 1: 8-byte copies)
+        const C* src = Tn + (((size_t)b << lML) + m0) * P;
+        for (int idx = tid; idx < (MS << LP); idx += nthr) cp_async_elem(tile + (idx >> LP) * LD + (idx & (P - 1)), src + idx);
+        if (stage_L) {
+            const C* Lb = LL + (size_t)b * Q * P;
+            constexpr int V = 16 / sizeof(C);
+            for (int idx = tid; idx < Q * P / V; idx += nthr) cp_async<16>(Lsm + idx * V, Lb + idx * V);
+        }
+    }
     cp_async_wait_all();
     __syncthreads();
 
-    // L2T + POST: thread owns one p and a group of MG consecutive m (L^L read once per q).
-    constexpr int MG = 8;
-    const int ngrp = (MS + MG - 1) / MG;
-    for (int idx = tid; idx < P * ngrp; idx += nthr) {
+    // L2T + POST: thread (p, g) owns one p and MG consecutive m (L^L read once per q, the MG
+    // L2T coefficients as two 16-byte broadcasts). MS * P / MG pairs, a multiple of nthr.
+    const C* Lb = LL + (size_t)b * Q * P;
+    for (int idx = tid; idx < (MS << LP) / MG; idx += nthr) {
         const int p = idx & (P - 1), g = idx >> LP;
         if (p == 0) continue;                                      // C_0 = I (R1)
         C acc[MG];
 #pragma unroll
         for (int u = 0; u < MG; ++u) acc[u] = zero<C>();
+        const R* a = s2m_sm + g * MG;
+#pragma unroll 4
         for (int q = 0; q < Q; ++q) {
             const C l = stage_L ? Lsm[q * P + p] : ldg_c(Lb + q * P + p);
+            R av[MG];
+            if constexpr (sizeof(R) == 4) {
+                const float4 a0 = *reinterpret_cast<const float4*>(a + q * MS), a1 = *reinterpret_cast<const float4*>(a + q * MS + 4);
+                av[0] = a0.x; av[1] = a0.y; av[2] = a0.z; av[3] = a0.w; av[4] = a1.x; av[5] = a1.y; av[6] = a1.z; av[7] = a1.w;
+            } else {
 #pragma unroll
-            for (int u = 0; u < MG; ++u)
-                if (g * MG + u < MS) rfma(acc[u], s2m_sm[q * MS + g * MG + u], l);
+                for (int u = 0; u < MG; u += 2) {
+                    const double2 d = *reinterpret_cast<const double2*>(a + q * MS + u);
+                    av[u] = d.x; av[u + 1] = d.y;
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < MG; ++u) rfma(acc[u], av[u], l);
         }
         const C rp = ldg_c(r + p), rh = ldg_c(rho + p);
 #pragma unroll
         for (int u = 0; u < MG; ++u) {
-            const int m = g * MG + u;
-            if (m < MS) {
-                C t = cadd(tile[m * LD + p], acc[u]);
-                t.x -= rp.y; t.y += rp.x;                           // + i r_p
-                tile[m * LD + p] = cmul(rh, t);
-            }
+            C* t = tile + (g * MG + u) * LD + p;
+            C v = cadd(*t, acc[u]);
+            v.x -= rp.y; v.y += rp.x;                               // + i r_p
+            *t = cmul(rh, v);
         }
     }
     __syncthreads();

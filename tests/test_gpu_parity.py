@@ -31,9 +31,9 @@ def F():
     return FmmFFT
 
 
-def run(F, N, P, B, Q, prec, M_L=64, G=1, virtual=False, seed=SI.DEFAULT_SEED):
+def run(F, N, P, B, Q, prec, M_L=64, G=1, virtual=False, seed=SI.DEFAULT_SEED, debug=False):
     x = SI.complex_uniform(0, N, seed=seed, dtype=NPDT[prec])
-    plan = F(N=N, P=P, G=G, B=B, Q=Q, precision=prec, M_L=M_L, virtual=virtual)
+    plan = F(N=N, P=P, G=G, B=B, Q=Q, precision=prec, M_L=M_L, virtual=virtual, debug=debug)
     xd = torch.from_numpy(x).cuda()
     y = plan(xd)
     torch.cuda.synchronize()
@@ -82,7 +82,7 @@ def test_cfg1_c128_matches_oracle_and_direct_dft(F):
 @pytest.mark.parametrize("prec", ["c64", "c128"])
 @pytest.mark.parametrize("N,P,B,Q,M_L", [(1 << 16, 16, 2, 16, 32), (1 << 18, 64, 3, 16, 64)])
 def test_stages_match_oracle(F, prec, N, P, B, Q, M_L):
-    plan, x, y = run(F, N, P, B, Q, prec, M_L)
+    plan, x, y = run(F, N, P, B, Q, prec, M_L, debug=True)
     L = O.tree_levels(N, P, M_L)
     S = x.astype(np.complex128).reshape(2 ** L, M_L, P)
     st = O.fmm_stages(S, N, P, B, Q)
