@@ -137,7 +137,7 @@ FMMFFT_API fmmfft_status_t fmmfft_stage_times(fmmfft_plan_t plan, float* ms, int
 FMMFFT_API const char* fmmfft_stage_name(int i);
 
 /* Internal buffers after an execute, for stage-by-stage parity tests. `which`:
- *   0 = T_near  [b][m][p]  (S2T output, N/G complex)
+ *   0 = T_near  [p][b][re/im][m]  (S2T output, N/G complex as 2N/G reals: p-major, planar per box)
  *   1 = M^l     [b][q][p]  (multipoles of level `level`, own boxes; slot p = FMM p)
  *   2 = L^l     [b][q][p]  (local expansions of level `level`, own boxes)
  *   3 = W       [k2][m]    (P-point FFT output before the transpose, N/G complex)

@@ -148,7 +148,7 @@ static const char* kStageNames[ST_COUNT + 1] = {"comm_S", "s2m", "m2m", "comm_M"
 
 struct RankBufs {
     int g = 0;
-    void* Tn = nullptr;      // [nb][M_L][P]   S2T output (T_near)
+    void* Tn = nullptr;      // [P][nb][2][M_L] S2T output (T_near, p-major, planar re/im per box)
     void* tmp = nullptr;     // M-FFT ping-pong buffer
     void* Sp = nullptr;      // S'[p][b][m]: p-major copy of the input for the tensor-core S2T
     void* W = nullptr;       // [k2][Mg]       P-FFT output = all-to-all send buffer
@@ -190,8 +190,9 @@ struct fmmfft_plan_s {
     std::vector<void*> m2l;          // by level
     std::vector<void*> m2l_pmaj;     // p-major copies for the fused per-p tree (G = 1), by level
     bool tree_p = false;             // use k_tree_p for the far field
+    int tree_cl = 1;                 // k_tree_pc: CTAs per FMM (cluster), 1 = not used
     bool tree_phased = false;        // ... as up / all-levels M2L / L2L-chain launches (FMMFFT_TREE=p) (k_tree_pq<.., false>, k_m2l_flat, k_tree_dn)
-    bool s2t_tc = false;             // S2T on tcgen05 (k_s2t_tc): complex64, M_L = 64, nb % 64 == 0
+    bool s2t_tc = false;             // S2T on tcgen05 (k_s2t_tc): complex64, M_L = 64, nb % 128 == 0
     void* toep = nullptr;            // its Toeplitz hi/lo operand table
     bool row_fft1 = false;           // M-point FFTs in one pass per row (k_fft_row), M fits smem
     void* twM = nullptr;             // its twiddles w_M^u, u < M/16
@@ -305,8 +306,8 @@ static fmmfft_status_t build_tables(fmmfft_plan_s* p) {
             if ((st = upload<R>(p, &p->m2l_pmaj[lev], tp))) return st;
         }
     }
-    // tensor-core S2T operand: Toep_p[i][k] = S2T_{p, (k - 64) - i}, split into tf32 hi + lo,
-    // in the UMMA K-major core-matrix layout [p][chunk][hi/lo][k4][r8][8][4] (kernel_s2t_tc.cuh)
+    // tensor-core S2T operator (kernel_s2t_tc.cuh): B_p[(s, i)][m] = S2T_{p, (s-1) 64 + m - i},
+    // split into tf32 hi + lo, UMMA K-major core-matrix layout [hi/lo][k4][r8][8][4] per p
     if (p->s2t_tc) {
         auto tf32 = [](double v) {                     // round to nearest (ties away), tf32 precision
             float f = (float)v;
@@ -317,22 +318,21 @@ static fmmfft_status_t build_tables(fmmfft_plan_s* p) {
             return f;
         };
         std::vector<float> tb((size_t)P * S2TC_TAB_FLOATS_PER_P, 0.f);
-        const int half = 64 * S2TC_CHUNK_K;                // floats of one of hi / lo per chunk
-        for (int pp = 1; pp < P; ++pp)
-            for (int c = 0; c < S2TC_NCHUNK; ++c)
-                for (int k4 = 0; k4 < S2TC_CHUNK_K / 4; ++k4)
-                    for (int i = 0; i < 64; ++i)
-                        for (int kk = 0; kk < 4; ++kk) {
-                            const int k = S2TC_CHUNK_K * c + 4 * k4 + kk;
-                            const long long d = (long long)(k - 64) - i;
-                            const double v = cotpi((double)(pp + (long long)P * d) / (double)N);
-                            const float hi = tf32(v);
-                            const float lo = tf32(v - (double)hi);
-                            const size_t base = (size_t)pp * S2TC_TAB_FLOATS_PER_P + (size_t)c * 2 * half;
-                            const size_t e = ((size_t)(k4 * 8 + (i >> 3)) * 8 + (i & 7)) * 4 + kk;
-                            tb[base + e] = hi;
-                            tb[base + half + e] = lo;
-                        }
+        const size_t half = S2TC_B_BYTES / 4;              // floats of one of hi / lo
+        for (int pp = 1; pp < P; ++pp) {
+            for (int k4 = 0; k4 < 16; ++k4)
+                for (int r = 0; r < S2TC_N; ++r)
+                    for (int kk = 0; kk < 4; ++kk) {
+                        const int seg = r / 64, i = r % 64, m = 4 * k4 + kk;
+                        const long long d = (long long)(seg - 1) * 64 + m - i;
+                        const double v = cotpi((double)(pp + (long long)P * d) / (double)N);
+                        const float hi = tf32(v);
+                        const float lo = tf32(v - (double)hi);
+                        const size_t e = (size_t)pp * S2TC_TAB_FLOATS_PER_P + ((size_t)k4 * (S2TC_N / 8) + r / 8) * 32 + (r % 8) * 4 + kk;
+                        tb[e] = hi;
+                        tb[e + half] = lo;
+                    }
+        }
         fmmfft_status_t st2 = dalloc(p, &p->toep, tb.size() * sizeof(float));
         if (st2) return st2;
         CUDA_TRY(cudaMemcpy(p->toep, tb.data(), tb.size() * sizeof(float), cudaMemcpyHostToDevice));
@@ -466,6 +466,10 @@ static fmmfft_status_t init_kernel_attrs() {
             set((const void*)k_tree_dn<16, 512>);
             set((const void*)k_tree_dn<8, 512>);
             set((const void*)k_tree_pq<8, 512, 8>);
+            set((const void*)k_tree_pc<16, 512, 2>);
+            set((const void*)k_tree_pc<16, 256, 4>);
+            set((const void*)k_tree_pc<8, 512, 2>);
+            set((const void*)k_tree_pc<8, 256, 4>);
         }
         if constexpr (sizeof(R) == 4) set((const void*)k_s2t_tc);
         set((const void*)k_tree_p<R, 1>);
@@ -497,6 +501,16 @@ static size_t tree_p_smem(const fmmfft_plan_s* p, int threads) {
     const size_t npyr = (((size_t)2 << p->L) - ((size_t)1 << p->B)) * Q;
     const size_t tabs = ((size_t)(1 << p->B) - 3) * Q * Q + (size_t)(p->L - p->B) * 4 * Q * Q;
     return npyr * p->esz + (4 * Q * Q + tabs) * p->rsz + 32 * p->esz;
+}
+
+// shared memory of k_tree_pc (cluster of CL CTAs per FMM)
+static size_t tree_pc_smem(const fmmfft_plan_s* p, int CL) {
+    const size_t Q = p->Q, QQ = Q * Q, nbB = (size_t)1 << p->B;
+    const size_t tabB = (nbB - 3) * QQ;
+    auto H = [&](int l) { return ((size_t)1 << l) / CL; };
+    size_t cplx = 32 + nbB * Q + (nbB / CL) * Q + H(p->L) * Q + (p->L > 0 ? H(p->L - 1) : 0) * Q;
+    for (int l = p->B + 1; l <= p->L; ++l) cplx += (H(l) + 6) * Q;
+    return (2 * QQ + tabB + (size_t)(p->L - p->B) * 4 * QQ) * 4 + QQ * 8 + cplx * 8;
 }
 
 // ------------------------------------------------------------------ execute
@@ -579,7 +593,7 @@ struct Exec {
                 constexpr int PCv = decltype(pc)::value;
                 if constexpr (!(sizeof(R) == 8 && PCv > 16))
                     launch_pdl(k_s2m<R, PCv>, grid, PCv * (Qp / 4) * nbx, smem, s, S, interior(rb.Mpad[p->L]), (const R*)p->s2mT, p->P,
-                                                                           p->M_L, p->Q, (C*)rb.Sp, p->nb, nbx);
+                                                                           p->M_L, p->Q, (C*)rb.Sp, (C*)rb.Tn, p->nb, nbx);
             });
             LAUNCH_CHECK();
         }
@@ -592,14 +606,13 @@ struct Exec {
                 CUDA_TRY(cudaEventRecord(p->fork2, s));             // needs S' from k_s2m
                 CUDA_TRY(cudaStreamWaitEvent(p->side, p->fork2, 0));
                 if ((st = mark_on(p->ev_s2t[0], p->side))) return st;
+                const int ntile = p->nb / S2TC_BOXES;
+                int tpc = 1;                                       // tiles per CTA: about one wave
+                while (tpc < ntile && (long long)(ntile / tpc) * (p->P - 1) > 148) tpc *= 2;
                 for (RankBufs& rb : p->ranks) {
-                    const C* S = in[p->virt ? rb.g : 0];
-                    const size_t box = (size_t)p->M_L * p->P;
-                    const C* hl = p->G == 1 ? S + (size_t)(p->nb - 1) * box : (const C*)rb.haloL;
-                    const C* hr = p->G == 1 ? S : (const C*)rb.haloR;
-                    const dim3 grid((unsigned)(p->nb / S2TC_BOXES), (unsigned)p->P);
-                    launch_pdl(k_s2t_tc, grid, 256, s2tc_smem_bytes(), p->side, (const C*)rb.Sp, S, hl, hr, (C*)rb.Tn,
-                                                                         (const float*)p->toep, p->P, p->nb, p->G);
+                    const dim3 grid((unsigned)((ntile + tpc - 1) / tpc), (unsigned)(p->P - 1));
+                    launch_pdl(k_s2t_tc, grid, S2TC_THREADS, s2tc_smem_bytes(), p->side, (const C*)rb.Sp, (const C*)rb.haloL,
+                               (const C*)rb.haloR, (float*)rb.Tn, (const float*)p->toep, p->P, p->nb, p->G, tpc);
                     LAUNCH_CHECK();
                 }
                 if ((st = mark_on(p->ev_s2t[1], p->side))) return st;
@@ -721,6 +734,19 @@ struct Exec {
                         else            launch_pdl(k_tree_dn<8, 512>, p->P - 1, 512, smem3, s, a, (const float*)p->m2m, p->P);
                         LAUNCH_CHECK();
                     }
+                    continue;
+                }
+                if (p->tree_cl > 1) {                            // cluster of CL CTAs per FMM (k_tree_pc)
+                    const size_t smem = tree_pc_smem(p, p->tree_cl);
+                    const unsigned grid = (unsigned)((p->P - 1) * p->tree_cl);
+                    if (p->tree_cl == 2) {
+                        if (p->Q == 16) launch_plain(k_tree_pc<16, 512, 2>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
+                        else            launch_plain(k_tree_pc<8, 512, 2>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
+                    } else {
+                        if (p->Q == 16) launch_plain(k_tree_pc<16, 256, 4>, grid, 256, smem, s, a, (const float*)p->m2m, p->P, tabB);
+                        else            launch_plain(k_tree_pc<8, 256, 4>, grid, 256, smem, s, a, (const float*)p->m2m, p->P, tabB);
+                    }
+                    LAUNCH_CHECK();
                     continue;
                 }
                 if ((p->Q == 16 || p->Q == 8) && (1LL << p->L) <= 8LL * ngrp) {
@@ -1166,15 +1192,21 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
         const size_t scratch = (((size_t)3 * Q) << (L > 0 ? L - 1 : 0)) * p->esz + (size_t)2 * Q * Q * p->rsz;
         p->tree_p = (G == 1) && ((long long)Q << L) <= 8LL * threads && tree_p_smem(p, threads) + scratch <= (size_t)optin;
         if (const char* e = getenv("FMMFFT_TREE")) {
-            p->tree_p = p->tree_p && (e[0] == 'p' || e[0] == 'f');
+            p->tree_p = p->tree_p && (e[0] == 'p' || e[0] == 'f' || e[0] == 'c');
             p->tree_phased = e[0] == 'p';
         }
+        // complex64, Q = 8 / 16: split each FMM's tree over a cluster of CL CTAs (k_tree_pc)
+        if (p->tree_p && !p->tree_phased && precision == FMMFFT_C64 && (Q == 16 || Q == 8)) {
+            int cl = 2;
+            if (const char* e = getenv("FMMFFT_TREE_CL")) cl = atoi(e);
+            if (const char* e = getenv("FMMFFT_TREE")) if (e[0] == 'f') cl = 1;
+            if ((cl == 2 || cl == 4) && (1 << B) >= cl && tree_pc_smem(p, cl) <= (size_t)optin) p->tree_cl = cl;
+        }
     }
-    // tensor-core S2T: correct (parity-tested) but not yet faster end to end than the FFMA2 SIMT
-    // kernel on this workload, so opt-in: FMMFFT_S2T=tc
-    p->s2t_tc = false;
-    if (const char* e = getenv("FMMFFT_S2T"))
-        p->s2t_tc = e[0] == 't' && precision == FMMFFT_C64 && M_L == 64 && (p->nb % S2TC_BOXES) == 0;
+    // tensor-core S2T (k_s2t_tc, 3xTF32 on tcgen05) for complex64 with M_L = 64 and whole 128-box
+    // tiles per rank; FMMFFT_S2T=simt selects the FFMA2 kernel (k_near_up) instead
+    p->s2t_tc = precision == FMMFFT_C64 && M_L == 64 && (p->nb % S2TC_BOXES) == 0;
+    if (const char* e = getenv("FMMFFT_S2T")) p->s2t_tc = p->s2t_tc && e[0] == 't';
     const char* g_env = getenv("FMMFFT_NO_GRAPH");
     p->use_graph = !(g_env && g_env[0] == '1');
     plan_radices(p);

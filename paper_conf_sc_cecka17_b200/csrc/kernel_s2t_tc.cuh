@@ -1,176 +1,251 @@
 // kernel_s2t_tc.cuh — S2T (Alg. 1 line 3, §4.6) on the 5th-generation tensor
 // cores, complex64, M_L = 64.
 //
-// For one FMM p and a tile of 64 consecutive leaf boxes b0..b0+63 the near field is the GEMM
-//     D[n][i] = sum_{k < 192} A[n][k] * Toep_p[i][k],     Toep_p[i][k] = S2T_{p, (k - 64) - i}
-// with rows n = 2 (b - b0) + c (box, re/im) — UMMA M = 128 — columns i < 64 (N = 64) and
-// k = the position in the window [box b-1, b, b+1] (K = 192, the paper's -M_L <= j < 2 M_L).
-// A[n][k] = S_{p, k mod 64, b - 1 + k div 64}.c is built in shared memory from the window of the
-// p-major copy S'[p][b][m] that k_s2m writes (one contiguous bulk copy per CTA); Toep_p is
-// precomputed per plan (fp64 -> tf32 hi/lo) in the UMMA K-major core-matrix layout and streamed
-// with cp.async.bulk. Precision: 3xTF32, D = Ahi Bhi + Ahi Blo + Alo Bhi
-// accumulated in fp32 in tensor memory (plain TF32 misses the 1e-5 bound).
-// K is processed in 12 chunks of 16, double-buffered; one thread issues the 6 MMAs of a chunk
-// (tcgen05.mma kind::tf32, M=128 N=64 K=8) and commits them to an mbarrier.
-// p = 0 (the identity, R1) is a plain copy by its own CTAs.
+// The near field of leaf box b for FMM p is
+//     T[b][i] = sum_{j=-64}^{127} K_p[j - i] S_window[j],   K_p[k] = cot(pi (p + P k) / N),
+// the window being boxes b-1, b, b+1. Split by source box (segment s = 0, 1, 2 <-> box b-1+s):
+//     T[b][i] = sum_{s<3} sum_{m<64} A[b - 1 + s][m] B_s[i][m],   B_s[i][m] = K_p[(s-1) 64 + m - i],
+// with A[b][m] = S_{p m b} (one real component at a time; the operator is real).
+// For a tile of 128 consecutive boxes this is three accumulating GEMMs (UMMA M = 128 boxes,
+// N = 64 outputs i, K = 64 points m) whose A operands are the SAME shared-memory rows shifted by
+// one box: A is stored K-major with 8-row core-matrix groups packed back to back (SBO = 128 B), so
+// row r sits at r x 16 bytes and "the rows of boxes b0-1+s .. b0+126+s" is the descriptor of row
+// s — a 16-byte offset. The A buffer holds 130 rows (boxes b0-1 .. b0+128): the data is used once,
+// never Toeplitz-expanded, and the accumulator already holds T (no shift in the epilogue).
+// B_s is the per-p Toeplitz operator, precomputed per plan in fp64 and split into tf32 hi + lo.
+// Precision: 3xTF32, T = Ahi Bhi + Ahi Blo + Alo Bhi accumulated in fp32 in tensor memory (plain
+// TF32 misses the 1e-5 bound): 9 MMAs (M=128, N=64, K=8) per K step and component.
+//
+// CTA = (FMM p, run of 128-box tiles), warp-specialised, 9 warps:
+//   warps 0-3  build A (re/im x hi/lo, K chunks of 16 in a 2-slot ring) from the p-major copy
+//              S'[p][b][m] (the next chunk prefetched into registers); halo rows from the
+//              neighbouring boxes (periodic wrap at G = 1, the halo buffers at rank edges);
+//   warp 8     loads the operator B_p (bulk copies, one mbarrier per K chunk) and issues the MMAs,
+//              committing each chunk's MMAs to the slot's mbarrier;
+//   warps 4-7  (TMEM lane quarters 0-3) the epilogue: tcgen05.ld of T (re and im accumulators),
+//              coalesced stores through a 32 x 32 shared-memory transpose per warp.
+// Two TMEM accumulator pairs (2 x 128 columns): the epilogue of tile t overlaps the MMAs of t+1.
+// Output T_near is p-major and planar per box: [p][b][re/im][m] (what k_post_pfft reads).
+// p = 0 (the identity, R1) is written by k_s2m.
 #pragma once
 #include "common.cuh"
 #include "tcgen05.cuh"
 
+#ifndef STAMP
+#define STAMP(i) do {} while (0)                          // timing probes (scripts/micro/bench_s2t_tc.cu)
+#endif
+
 namespace fmmfft {
 
-constexpr int S2TC_BOXES = 64;                 // boxes per tile (UMMA M = 2 * 64)
-constexpr int S2TC_CHUNK_K = 16;               // K per pipeline chunk
-constexpr int S2TC_NCHUNK = 192 / S2TC_CHUNK_K;
-constexpr int S2TC_LBO_A = 2064;               // bytes between K-halves of A (2048 + 16: bank skew)
-constexpr int S2TC_A_BYTES = (S2TC_CHUNK_K / 4) * S2TC_LBO_A;   // one of hi / lo
-constexpr int S2TC_B_BYTES = 64 * S2TC_CHUNK_K * 4;   // one of hi / lo, LBO 1024, SBO 128
-constexpr int S2TC_TAB_FLOATS_PER_P = S2TC_NCHUNK * 2 * 64 * S2TC_CHUNK_K;   // [chunk][hi,lo][k4][r8][8][4]
+constexpr int S2TC_BOXES = 128;                           // boxes per tile (UMMA M)
+constexpr int S2TC_ROWS = S2TC_BOXES + 2;                 // + halo boxes b0-1, b0+128
+constexpr int S2TC_KC = 16;                               // K (m) per A chunk
+constexpr int S2TC_NKC = 64 / S2TC_KC;
+constexpr int S2TC_LBO_A = S2TC_ROWS * 16;                // bytes between k4 columns of A (2080)
+constexpr int S2TC_A_PART = (S2TC_KC / 4) * S2TC_LBO_A;   // one (component, hi/lo) part of a chunk
+constexpr int S2TC_A_SLOT = 4 * S2TC_A_PART;              // [re/im][hi/lo] parts
+constexpr int S2TC_N = 192;                               // operator rows (segment, i)
+constexpr int S2TC_B_K4 = (S2TC_N / 8) * 128;             // bytes per k4 column of B (24 core matrices)
+constexpr int S2TC_B_BYTES = 16 * S2TC_B_K4;              // one of hi / lo (K = 64)
+constexpr int S2TC_TAB_FLOATS_PER_P = 2 * S2TC_B_BYTES / 4;   // [hi,lo][k4 16][r8 24][8][4]
+constexpr int S2TC_THREADS = 288;
 
-constexpr int S2TC_SCOL_BYTES = ((S2TC_BOXES + 2) * 64 * 8 + 1023) / 1024 * 1024;   // staged S column
-__host__ __device__ constexpr size_t s2tc_smem_bytes() {
-    return (size_t)S2TC_SCOL_BYTES                       // staged S column (66 boxes x 64 m, float2)
-           + 2 * (2 * S2TC_A_BYTES)                      // A hi/lo, double-buffered
-           + 2 * (2 * S2TC_B_BYTES)                      // B hi/lo, double-buffered
-           + 64;                                         // mbarriers + TMEM address
-}
+struct S2tcSmem {                                         // byte offsets
+    static constexpr int B = 0;
+    static constexpr int A = B + 2 * S2TC_B_BYTES;              // 2-slot ring of K chunks
+    static constexpr int XT = A + 2 * S2TC_A_SLOT;              // per-warp transpose [4][32][33] floats
+    static constexpr int BAR = XT + 4 * 32 * 33 * 4;            // 12 mbarriers
+    static constexpr int TSLOT = BAR + 12 * 8;
+    static constexpr int TOTAL = TSLOT + 16;
+};
+__host__ __device__ constexpr size_t s2tc_smem_bytes() { return (size_t)S2tcSmem::TOTAL; }
 
-__global__ void __launch_bounds__(256, 2)
-k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ S, const float2* __restrict__ haloL,
-         const float2* __restrict__ haloR, float2* __restrict__ Tn, const float* __restrict__ toep, int P, int nb, int G) {
+__global__ void __launch_bounds__(S2TC_THREADS, 1)
+k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const float2* __restrict__ haloR,
+         float* __restrict__ Tn, const float* __restrict__ toep, int P, int nb, int G, int tiles_per_cta) {
     pdl_trigger();
     pdl_wait();
+    STAMP(0);
     extern __shared__ __align__(1024) unsigned char smem_tc[];
-    float2* Scol = reinterpret_cast<float2*>(smem_tc);                           // [66][64]
-    unsigned char* Abase = smem_tc + S2TC_SCOL_BYTES;                            // 2 x (hi, lo)
-    unsigned char* Bbase = Abase + 2 * 2 * S2TC_A_BYTES;                          // 2 x (hi, lo)
-    uint64_t* bar = reinterpret_cast<uint64_t*>(Bbase + 2 * 2 * S2TC_B_BYTES);    // [0,1] B load, [2,3] mma, [4] S
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 5);
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int b0 = blockIdx.x * S2TC_BOXES;
-    const int p = blockIdx.y;
-    const size_t box = (size_t)64 * P;
+    unsigned char* Bsm = smem_tc + S2tcSmem::B;
+    unsigned char* Asm = smem_tc + S2tcSmem::A;
+    float* Xt = reinterpret_cast<float*>(smem_tc + S2tcSmem::XT);
+    uint64_t* bar = reinterpret_cast<uint64_t*>(smem_tc + S2tcSmem::BAR);
+    uint64_t* bfull = bar;                                       // [4] operator chunk landed
+    uint64_t* cfull = bar + 4;                                   // [2] A slot built (128 arrivals)
+    uint64_t* cempty = bar + 6;                                  // [2] MMAs of A slot done (commit)
+    uint64_t* afull = bar + 8;                                   // [2] accumulators complete (commit)
+    uint64_t* aempty = bar + 10;                                 // [2] accumulators read (128 arrivals)
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(smem_tc + S2tcSmem::TSLOT);
 
-    if (p == 0) {                                                // C_0 = I: T[., ., 0] = S[., ., 0]
-        for (int o = tid; o < S2TC_BOXES * 64; o += blockDim.x)
-            Tn[((size_t)b0 * 64 + o) * P] = S[((size_t)b0 * 64 + o) * P];
-        return;
-    }
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int p = blockIdx.y + 1;
+    const int ntile = nb / S2TC_BOXES;
+    const int t0 = blockIdx.x * tiles_per_cta;
+    const int t1 = min(ntile, t0 + tiles_per_cta);
+    if (t0 >= t1) return;
+    const int nit = t1 - t0;
+    const size_t pblk = (size_t)nb * 64;                         // elements per p block of S' / T
+    const float2* spp = Sp + (size_t)p * pblk;
+
     if (tid == 0) {
-        for (int k = 0; k < 5; ++k) tc::mbar_init(&bar[k], 1);
+        for (int k = 0; k < 12; ++k) tc::mbar_init(&bar[k], (k == 4 || k == 5 || k >= 10) ? 128u : 1u);
         tc::fence_barrier_init();
     }
-    if (warp == 0) tc::tmem_alloc<64>(tmem_slot);
+    if (warp == 0) tc::tmem_alloc<256>(tmem_slot);
     tc::tc_fence_before();
     __syncthreads();
     tc::tc_fence_after();
     const uint32_t tmem = *tmem_slot;
-    const float* tp = toep + (size_t)p * S2TC_TAB_FLOATS_PER_P;
-    const float2* spp = Sp + (size_t)p * nb * 64;                // S'[p][b][m]
-    // window boxes b0-1 .. b0+64: the interior ones in one bulk copy from S'
-    const int ilo = max(b0 - 1, 0), ihi = min(b0 + S2TC_BOXES + 1, nb);   // [ilo, ihi)
-    if (tid == 0) {
-        tc::mbar_expect_tx(&bar[4], (uint32_t)(ihi - ilo) * 512);
-        tc::bulk_g2s(Scol + (ilo - (b0 - 1)) * 64, spp + (size_t)ilo * 64, (uint32_t)(ihi - ilo) * 512, &bar[4]);
-        for (int c = 0; c < 2; ++c) {                            // B chunks 0 and 1
-            tc::mbar_expect_tx(&bar[c], 2 * S2TC_B_BYTES);
-            tc::bulk_g2s(Bbase + c * 2 * S2TC_B_BYTES, tp + (size_t)c * 2 * 64 * S2TC_CHUNK_K, 2 * S2TC_B_BYTES, &bar[c]);
-        }
-    }
-    // edge boxes -1 / nb: neighbour halos (G > 1) or the periodic wrap (G = 1)
-    if (b0 == 0 || b0 + S2TC_BOXES == nb) {
-        for (int o = tid; o < 2 * 64; o += blockDim.x) {
-            const int side = o >> 6, m = o & 63;
-            const int bb = side ? b0 + S2TC_BOXES : b0 - 1;
-            if (bb >= 0 && bb < nb) continue;
-            const int u = bb - (b0 - 1);
-            if (G == 1) Scol[u * 64 + m] = spp[(size_t)(bb < 0 ? nb - 1 : 0) * 64 + m];
-            else Scol[u * 64 + m] = (bb < 0 ? haloL : haloR)[(size_t)m * P + p];
-        }
-    }
-    tc::mbar_wait(&bar[4], 0);
-    __syncthreads();
-    (void)box;
+    STAMP(1);
 
-    constexpr uint32_t IDESC = tc::idesc_tf32(128, 64);
-    for (int c = 0; c < S2TC_NCHUNK; ++c) {
-        const int buf = c & 1;
-        unsigned char* Ahi = Abase + buf * 2 * S2TC_A_BYTES;
-        unsigned char* Alo = Ahi + S2TC_A_BYTES;
-        unsigned char* Bhi = Bbase + buf * 2 * S2TC_B_BYTES;
-        unsigned char* Blo = Bhi + S2TC_B_BYTES;
-        if (c >= 2) {
-            tc::mbar_wait(&bar[2 + buf], ((c - 2) >> 1) & 1);    // MMAs of chunk c-2 done: buffers free
-            if (tid == 0) {
-                tc::mbar_expect_tx(&bar[buf], 2 * S2TC_B_BYTES);
-                tc::bulk_g2s(Bhi, tp + (size_t)c * 2 * 64 * S2TC_CHUNK_K, 2 * S2TC_B_BYTES, &bar[buf]);
-            }
-        }
-        // build A chunk c: rows n = 2 bl + cc, K columns kk = 4 k4 + j (window k = 16 c + kk)
-        const int kb = (S2TC_CHUNK_K * c) >> 6;                  // window box offset 0, 1, 2
-        const int m0 = (S2TC_CHUNK_K * c) & 63;
-        {
-            const int k4 = tid & 3, bl = tid >> 2;               // 64 boxes x 4 k4
-            const float4* sp = reinterpret_cast<const float4*>(Scol + (bl + kb) * 64 + m0 + 4 * k4);
-            const float4 u0 = sp[0], u1 = sp[1];                 // (re, im) of 4 consecutive m
-            const float re[4] = {u0.x, u0.z, u1.x, u1.z}, im[4] = {u0.y, u0.w, u1.y, u1.w};
-            float4 rh, rl, ih, il;
-            float* prh = &rh.x; float* prl = &rl.x; float* pih = &ih.x; float* pil = &il.x;
+    if (warp < 4) {
+        // ------------------------------------------------------------ A builders (128 threads)
+        // item j: row r = idx >> 2 (box b0 - 1 + r), k4 = idx & 3, idx = tid + 128 j < 4 x 130
+        constexpr int NJ = (4 * S2TC_ROWS + 127) / 128;          // 5
+        float4 sv[NJ][2];
+        auto load_chunk = [&](int t, int kc) {
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                const float h1 = tc::to_tf32(re[j]); prh[j] = h1; prl[j] = re[j] - h1;
-                const float h2 = tc::to_tf32(im[j]); pih[j] = h2; pil[j] = im[j] - h2;
+            for (int j = 0; j < NJ; ++j) {
+                const int idx = tid + 128 * j;
+                if (idx < 4 * S2TC_ROWS) {
+                    const int r = idx >> 2, k4 = idx & 3;
+                    const int g = t * S2TC_BOXES - 1 + r;        // global box (within this rank)
+                    const int m = S2TC_KC * kc + 4 * k4;
+                    if (g >= 0 && g < nb) {
+                        const float4* src = reinterpret_cast<const float4*>(spp + (size_t)g * 64 + m);
+                        sv[j][0] = __ldg(src);
+                        sv[j][1] = __ldg(src + 1);
+                    } else if (G == 1) {                         // periodic wrap (R8)
+                        const float4* src = reinterpret_cast<const float4*>(spp + (size_t)((g + nb) % nb) * 64 + m);
+                        sv[j][0] = __ldg(src);
+                        sv[j][1] = __ldg(src + 1);
+                    } else {                                     // neighbour rank's box ([m][P] layout)
+                        const float2* h = (g < 0 ? haloL : haloR) + (size_t)m * P + p;
+                        const float2 a = __ldg(h), b = __ldg(h + P), c = __ldg(h + 2 * P), d = __ldg(h + 3 * P);
+                        sv[j][0] = make_float4(a.x, a.y, b.x, b.y);
+                        sv[j][1] = make_float4(c.x, c.y, d.x, d.y);
+                    }
+                }
             }
-            const int n = 2 * bl;                                // re row; im row = n + 1
-            const int offr = k4 * S2TC_LBO_A + (n >> 3) * 128 + (n & 7) * 16;
-            *reinterpret_cast<float4*>(Ahi + offr) = rh;
-            *reinterpret_cast<float4*>(Alo + offr) = rl;
-            *reinterpret_cast<float4*>(Ahi + offr + 16) = ih;
-            *reinterpret_cast<float4*>(Alo + offr + 16) = il;
+        };
+        load_chunk(t0, 0);
+        for (int it = 0; it < nit; ++it) {
+            for (int kc = 0; kc < S2TC_NKC; ++kc) {
+                const int gi = it * S2TC_NKC + kc, slot = gi & 1, use = gi >> 1;
+                if (use > 0) tc::mbar_wait(&cempty[slot], (use - 1) & 1);   // MMAs done with this slot
+                unsigned char* As = Asm + slot * S2TC_A_SLOT;
+#pragma unroll
+                for (int j = 0; j < NJ; ++j) {
+                    const int idx = tid + 128 * j;
+                    if (idx < 4 * S2TC_ROWS) {
+                        const int r = idx >> 2, k4 = idx & 3;
+                        const float4 u0 = sv[j][0], u1 = sv[j][1];   // (re, im) of 4 consecutive m
+                        const float re[4] = {u0.x, u0.z, u1.x, u1.z}, im[4] = {u0.y, u0.w, u1.y, u1.w};
+                        float4 rh, rl, ihv, il;
+                        float* prh = &rh.x; float* prl = &rl.x; float* pih = &ihv.x; float* pil = &il.x;
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) {
+                            const float h1 = tc::to_tf32(re[q]); prh[q] = h1; prl[q] = re[q] - h1;
+                            const float h2 = tc::to_tf32(im[q]); pih[q] = h2; pil[q] = im[q] - h2;
+                        }
+                        const int off = k4 * S2TC_LBO_A + r * 16;   // [c][hi/lo][k4][row][16 B]
+                        *reinterpret_cast<float4*>(As + 0 * S2TC_A_PART + off) = rh;
+                        *reinterpret_cast<float4*>(As + 1 * S2TC_A_PART + off) = rl;
+                        *reinterpret_cast<float4*>(As + 2 * S2TC_A_PART + off) = ihv;
+                        *reinterpret_cast<float4*>(As + 3 * S2TC_A_PART + off) = il;
+                    }
+                }
+                tc::fence_proxy_async();
+                tc::mbar_arrive(&cfull[slot]);
+                if (it < 2) STAMP(41 + 4 * it + kc);
+                // prefetch the next chunk (next tile's first chunk after the last one)
+                if (kc + 1 < S2TC_NKC) load_chunk(t0 + it, kc + 1);
+                else if (it + 1 < nit) load_chunk(t0 + it + 1, 0);
+            }
         }
-        tc::fence_proxy_async();
-        __syncthreads();
-        if (tid == 0) {
-            tc::mbar_wait(&bar[buf], (c >> 1) & 1);              // B chunk landed
+    } else if (warp == 8) {
+        // ------------------------------------------------------------ operator loads + MMA issue
+        if (lane == 0) {
+            const float* tp = toep + (size_t)p * S2TC_TAB_FLOATS_PER_P;
+            for (int kc = 0; kc < S2TC_NKC; ++kc) {              // B chunk kc: k4 in [4 kc, 4 kc + 4), hi and lo
+                tc::mbar_expect_tx(&bfull[kc], 2 * 4 * S2TC_B_K4);
+                tc::bulk_g2s(Bsm + kc * 4 * S2TC_B_K4, tp + kc * S2TC_B_K4, 4 * S2TC_B_K4, &bfull[kc]);
+                tc::bulk_g2s(Bsm + S2TC_B_BYTES + kc * 4 * S2TC_B_K4, tp + S2TC_B_BYTES / 4 + kc * S2TC_B_K4,
+                             4 * S2TC_B_K4, &bfull[kc]);
+            }
+            constexpr uint32_t IDESC = tc::idesc_tf32(128, 64);
+            for (int it = 0; it < nit; ++it) {
+                const int buf = it & 1;
+                if (it >= 2) tc::mbar_wait(&aempty[buf], ((it >> 1) + 1) & 1);   // epilogue of tile it-2 done
+                for (int kc = 0; kc < S2TC_NKC; ++kc) {
+                    const int gi = it * S2TC_NKC + kc, slot = gi & 1, use = gi >> 1;
+                    if (it == 0) tc::mbar_wait(&bfull[kc], 0);
+                    tc::mbar_wait(&cfull[slot], use & 1);
+                    tc::tc_fence_after();
+                    const unsigned char* As = Asm + slot * S2TC_A_SLOT;
+#pragma unroll
+                    for (int st = 0; st < S2TC_KC / 8; ++st) {
+                        const unsigned char* bk = Bsm + (4 * kc + 2 * st) * S2TC_B_K4;
+#pragma unroll
+                        for (int c = 0; c < 2; ++c) {
+                            const uint32_t d = tmem + (uint32_t)(buf * 128 + c * 64);
+                            const unsigned char* ahp = As + (2 * c) * S2TC_A_PART + 2 * st * S2TC_LBO_A;
+                            const unsigned char* alp = As + (2 * c + 1) * S2TC_A_PART + 2 * st * S2TC_LBO_A;
+#pragma unroll
+                            for (int s = 0; s < 3; ++s) {        // rows of boxes b0-1+s ..: 16-byte offset
+                                const uint64_t ah = tc::umma_desc_kmajor(ahp + 16 * s, S2TC_LBO_A, 128);
+                                const uint64_t al = tc::umma_desc_kmajor(alp + 16 * s, S2TC_LBO_A, 128);
+                                const uint64_t bh = tc::umma_desc_kmajor(bk + s * 1024, S2TC_B_K4, 128);
+                                const uint64_t blo = tc::umma_desc_kmajor(bk + S2TC_B_BYTES + s * 1024, S2TC_B_K4, 128);
+                                tc::mma_tf32(d, ah, bh, IDESC, (kc | st | s) ? 1u : 0u);
+                                tc::mma_tf32(d, ah, blo, IDESC, 1u);
+                                tc::mma_tf32(d, al, bh, IDESC, 1u);
+                            }
+                        }
+                    }
+                    tc::mma_commit(&cempty[slot]);
+                    if (it < 2) STAMP(2 + 4 * it + kc);
+                }
+                tc::mma_commit(&afull[buf]);
+            }
+        }
+    } else {
+        // ------------------------------------------------------------ epilogue (warps 4-7)
+        // warp q reads TMEM lanes 32 q .. 32 q + 31 = boxes b0 + 32 q + lane
+        const int q = warp & 3;
+        float* xt = Xt + q * 32 * 33;
+        for (int it = 0; it < nit; ++it) {
+            const int t = t0 + it, buf = it & 1;
+            if (it < 4) STAMP(20 + 4 * it);
+            tc::mbar_wait(&afull[buf], (it >> 1) & 1);
             tc::tc_fence_after();
+            if (it < 4) STAMP(21 + 4 * it);
+            // planar [p][b][c][m]: rows of boxes b0 + 32 q + r, r < 32
+            float* tw = Tn + ((size_t)p * nb + (size_t)t * S2TC_BOXES + 32 * q) * 128;
+#pragma unroll 1
+            for (int ch = 0; ch < 4; ++ch) {                     // (component, i half)
+                const int c = ch >> 1, h = ch & 1;
+                float v[32];
+                tc::tmem_ld32(tmem + ((uint32_t)(32 * q) << 16) + (uint32_t)(buf * 128 + c * 64 + 32 * h), v);
+                if (ch == 3) {                                   // accumulators free for tile it + 2
+                    tc::tc_fence_before();
+                    tc::mbar_arrive(&aempty[buf]);
+                }
 #pragma unroll
-            for (int st = 0; st < S2TC_CHUNK_K / 8; ++st) {
-                const uint64_t ah = tc::umma_desc_kmajor(Ahi + 2 * st * S2TC_LBO_A, S2TC_LBO_A, 128);
-                const uint64_t al = tc::umma_desc_kmajor(Alo + 2 * st * S2TC_LBO_A, S2TC_LBO_A, 128);
-                const uint64_t bh = tc::umma_desc_kmajor(Bhi + 2 * st * 1024, 1024, 128);
-                const uint64_t bl_ = tc::umma_desc_kmajor(Blo + 2 * st * 1024, 1024, 128);
-                const uint32_t acc0 = (c | st) ? 1u : 0u;
-                tc::mma_tf32(tmem, ah, bh, IDESC, acc0);
-                tc::mma_tf32(tmem, ah, bl_, IDESC, 1u);
-                tc::mma_tf32(tmem, al, bh, IDESC, 1u);
-            }
-            tc::mma_commit(&bar[2 + buf]);
-        }
-        __syncwarp();
-    }
-    tc::mbar_wait(&bar[2 + ((S2TC_NCHUNK - 1) & 1)], ((S2TC_NCHUNK - 1) >> 1) & 1);
-    tc::tc_fence_after();
-    // epilogue: warps w and w+4 read TMEM lanes 32 (w mod 4) .. +31, columns [32 (w / 4), +32)
-    {
-        const int q = warp & 3, half = warp >> 2;
-        float v[32];
-        tc::tmem_ld32(tmem + ((uint32_t)(32 * q) << 16) + 32 * half, v);
-        const int n = 32 * q + lane, bl = n >> 1;
-        const bool is_re = (lane & 1) == 0;
-        float2* trow = Tn + ((size_t)(b0 + bl) * 64) * P + p;
+                for (int k = 0; k < 32; ++k) xt[lane * 33 + k] = v[k];
+                __syncwarp();
 #pragma unroll
-        for (int k = 0; k < 32; ++k) {
-            const float other = __shfl_xor_sync(0xffffffffu, v[k], 1);
-            // even lane writes columns k < 16 of the pair, odd lane k >= 16
-            if ((k < 16) == is_re) {
-                const int i = 32 * half + k;
-                trow[(size_t)i * P] = is_re ? make_float2(v[k], other) : make_float2(other, v[k]);
+                for (int r = 0; r < 32; ++r) tw[(size_t)r * 128 + c * 64 + 32 * h + lane] = xt[r * 33 + lane];
+                __syncwarp();
             }
+            if (it < 4) STAMP(22 + 4 * it);
         }
     }
     tc::tc_fence_before();
     __syncthreads();
-    if (warp == 0) tc::tmem_dealloc<64>(tmem);
+    STAMP(40);
+    if (warp == 0) tc::tmem_dealloc<256>(tmem);
 }
 
 }  // namespace fmmfft

@@ -167,9 +167,13 @@ k_post_pfft(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2
     fill_twiddles<R>(tw, LP);
     pdl_wait();                                                   // T_near / L^L / r from the FMM stages
     {
-        // T_near rows [m][p] (contiguous P per m) -> tile rows (stride P + 1: 8-byte copies)
-        const C* src = Tn + (((size_t)b << lML) + m0) * P;
-        for (int idx = tid; idx < (MS << LP); idx += nthr) cp_async_elem(tile + (idx >> LP) * LD + (idx & (P - 1)), src + idx);
+        // T_near [p][b][re/im][m] (p blocks of 2 nb M_L = 2 Mg reals) -> tile [m][p] (stride P + 1)
+        const R* src = reinterpret_cast<const R*>(Tn) + ((size_t)b << (lML + 1)) + m0;
+        for (int idx = tid; idx < (MS << LP); idx += nthr) {
+            const int pp = idx >> lMS, m = idx & (MS - 1);
+            cp_async_elem(&tile[m * LD + pp].x, src + (size_t)pp * 2 * Mg + m);
+            cp_async_elem(&tile[m * LD + pp].y, src + (size_t)pp * 2 * Mg + M_L + m);
+        }
         if (stage_L) {
             const C* Lb = LL + (size_t)b * Q * P;
             constexpr int V = 16 / sizeof(C);

@@ -1,5 +1,5 @@
 // tcgen05.cuh — thin inline-PTX wrappers for the sm_100a tensor-core path (tcgen05 MMA with
-// accumulators in tensor memory, bulk async copies, mbarriers). Only what k_s2t_tc needs.
+// accumulators in tensor memory, bulk async copies, mbarriers, named barriers).
 #pragma once
 #include <stdint.h>
 
@@ -23,6 +23,13 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
         "@!P1 bra WAIT_%=;\n\t}\n" ::"r"(smem_u32(bar)),
         "r"(phase)
         : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(bar)) : "memory");
+}
+// named barrier for a subset of the CTA's warps (id 1..15, nthreads a multiple of 32)
+__device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
+    asm volatile("bar.sync %0, %1;\n" ::"r"(id), "r"(nthreads) : "memory");
 }
 __device__ __forceinline__ void fence_barrier_init() { asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory"); }
 // make generic-proxy shared-memory writes visible to the async proxy (tensor core, bulk copies)
@@ -93,6 +100,19 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
 #pragma unroll
     for (int k = 0; k < 32; ++k) v[k] = __uint_as_float(r[k]);
 }
+
+// 32 lanes x 16 columns of 32-bit TMEM -> 16 registers per thread
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, float* v) {
+    uint32_t r[16];
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];\n"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]),
+          "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+        : "r"(taddr));
+#pragma unroll
+    for (int k = 0; k < 16; ++k) v[k] = __uint_as_float(r[k]);
+}
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory"); }
 
 // round-to-nearest tf32 (kept in an f32 container)
 __device__ __forceinline__ float to_tf32(float x) {

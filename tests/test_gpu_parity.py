@@ -40,6 +40,13 @@ def run(F, N, P, B, Q, prec, M_L=64, G=1, virtual=False, seed=SI.DEFAULT_SEED, d
     return plan, x, y.cpu().numpy()
 
 
+def t_near(plan, P, L, M_L):
+    """T_near debug buffer ([p][b][re/im][m] reals) as complex [b][m][p]."""
+    t = plan.debug_buffer("T_near").cpu().numpy()
+    f = t.view(np.float32 if t.dtype == np.complex64 else np.float64).reshape(P, 2 ** L, 2, M_L)
+    return (f[:, :, 0, :] + 1j * f[:, :, 1, :]).astype(t.dtype).transpose(1, 2, 0)
+
+
 def rel(a, b):
     return O.rel_l2(np.asarray(a, dtype=np.complex128), b)
 
@@ -87,7 +94,7 @@ def test_stages_match_oracle(F, prec, N, P, B, Q, M_L):
     S = x.astype(np.complex128).reshape(2 ** L, M_L, P)
     st = O.fmm_stages(S, N, P, B, Q)
     tol = TOL_STAGE[prec]
-    Tn = plan.debug_buffer("T_near").cpu().numpy().reshape(2 ** L, M_L, P)
+    Tn = t_near(plan, P, L, M_L)
     assert rel(Tn, st["T_near"]) < tol
     assert np.array_equal(Tn[:, :, 0], S[:, :, 0].astype(Tn.dtype))        # p = 0 copies exactly
     for lev in range(B, L + 1):
@@ -215,8 +222,9 @@ def test_full_size_sampled(F, N, P, B, Q, prec, G):
 
 # ------------------------------------------------------------------ alternative kernel paths
 @pytest.mark.parametrize("env", [
-    {"FMMFFT_S2T": "tc"},        # S2T on tcgen05 (3xTF32, k_s2t_tc)
+    {"FMMFFT_S2T": "simt"},      # S2T on the FFMA2 SIMT kernel (k_near_up) instead of tcgen05
     {"FMMFFT_TREE": "f"},        # far field fused in one per-FMM kernel (k_tree_pq)
+    {"FMMFFT_TREE_CL": "4"},     # far field on a cluster of 4 CTAs per FMM (k_tree_pc)
     {"FMMFFT_TREE": "w"},        # far field as wide per-level kernels (k_up, k_base, k_tree_down)
     {"FMMFFT_NO_GRAPH": "1"},    # eager launches instead of a CUDA graph
     {"FMMFFT_ROWFFT": "0"},      # multi-pass M-point FFT (k_fft_pass) instead of k_fft_row
@@ -231,7 +239,7 @@ def test_alternative_paths(F, monkeypatch, env, N, P, B, Q, G):
     if G == 1:
         L = O.tree_levels(N, P, 64)
         st = O.fmm_stages(x.astype(np.complex128).reshape(2 ** L, 64, P), N, P, B, Q)
-        Tn = plan.debug_buffer("T_near").cpu().numpy().reshape(2 ** L, 64, P)
+        Tn = t_near(plan, P, L, 64)
         assert rel(Tn, st["T_near"]) < TOL_STAGE[prec]
         assert np.array_equal(Tn[:, :, 0], x.reshape(2 ** L, 64, P)[:, :, 0])
         LL = plan.debug_buffer("L", L).cpu().numpy().reshape(2 ** L, Q, P)
