@@ -118,6 +118,23 @@ static cudaError_t launch_plain(void (*kern)(KArgs...), dim3 grid, dim3 block, s
     return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
 }
 
+// Launch of a kernel with compile-time cluster dimensions, asking the scheduler to spread the
+// cluster's CTAs over distinct SMs (small CTAs would otherwise be packed onto one SM).
+template <typename... KArgs, typename... Args>
+static cudaError_t launch_cluster(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args&&... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterSchedulingPolicyPreference;
+    at[0].val.clusterSchedulingPolicyPreference = cudaClusterSchedulingPolicySpread;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
+
 // ------------------------------------------------------------------ communicator
 struct Comm {
     ncclComm_t comm = nullptr;
@@ -195,6 +212,7 @@ struct fmmfft_plan_s {
     bool s2t_tc = false;             // S2T on tcgen05 (k_s2t_tc): complex64, M_L = 64, nb % 128 == 0
     void* toep = nullptr;            // its Toeplitz hi/lo operand table
     bool row_fft1 = false;           // M-point FFTs in one pass per row (k_fft_row), M fits smem
+    int row_cl = 0;                  // ... on a cluster of row_cl CTAs per row (k_fft_rowc), 0 = off
     void* twM = nullptr;             // its twiddles w_M^u, u < M/16
     std::vector<fmmfft::RankBufs> ranks;
     std::vector<int> radices;        // M-FFT passes
@@ -345,7 +363,7 @@ static fmmfft_status_t build_tables(fmmfft_plan_s* p) {
         rho[2 * pp + 1] = pp ? -std::sin(M_PI * pp / P) * sn : 0.0;
     }
     if ((st = upload<R>(p, &p->rho, rho))) return st;
-    if (p->row_fft1) {                                   // w_M^u = exp(-2 pi i u / M), u < M/16
+    if (p->row_fft1 || p->row_cl) {                      // w_M^u = exp(-2 pi i u / M), u < M/16
         std::vector<double> tw(2 * (p->M / 16));
         for (long long u = 0; u < p->M / 16; ++u) {
             tw[2 * u] = std::cos(2 * M_PI * (double)u / (double)p->M);
@@ -485,6 +503,14 @@ static fmmfft_status_t init_kernel_attrs() {
             });
         for (int lr = 1; lr <= 10; ++lr)
             dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10>(lr, [&](auto v) { set((const void*)k_fft_pass<R, decltype(v)::value>); });
+        for (int lk = 8; lk <= kRowFftMax<R> - 1; ++lk)
+            dispatch<8, 9, 10, 11, 12, 13>(lk, [&](auto v) {
+                constexpr int LK = decltype(v)::value;
+                if constexpr (LK <= kRowFftMax<R> - 1) {
+                    set((const void*)k_fft_rowc<R, LK, 2>);
+                    set((const void*)k_fft_rowc<R, LK, 4>);
+                }
+            });
         for (int ll = 8; ll <= kRowFftMax<R>; ++ll)
             dispatch<8, 9, 10, 11, 12, 13, 14>(ll, [&](auto v) {
                 if constexpr (decltype(v)::value <= kRowFftMax<R>) set((const void*)k_fft_row<R, decltype(v)::value>);
@@ -587,7 +613,7 @@ struct Exec {
             const C* S = in[p->virt ? rb.g : 0];
             const int Qp = (p->Q + 3) / 4 * 4;
             const int nbx = p->nb >= 2 ? 2 : 1;                // boxes per CTA (k_s2m NBX = 2; nb is even or 1)
-            const size_t smem = (size_t)2 * p->M_L * PCs * sizeof(C) + (size_t)Qp * p->M_L * sizeof(R);
+            const size_t smem = (size_t)2 * p->M_L * (PCs + 1) * sizeof(C) + (size_t)Qp * p->M_L * sizeof(R);
             const dim3 grid((unsigned)(p->nb / nbx), (unsigned)(p->P / PCs));
             dispatch<2, 4, 8, 16, 32>(PCs, [&](auto pc) {
                 constexpr int PCv = decltype(pc)::value;
@@ -740,11 +766,11 @@ struct Exec {
                     const size_t smem = tree_pc_smem(p, p->tree_cl);
                     const unsigned grid = (unsigned)((p->P - 1) * p->tree_cl);
                     if (p->tree_cl == 2) {
-                        if (p->Q == 16) launch_plain(k_tree_pc<16, 512, 2>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
-                        else            launch_plain(k_tree_pc<8, 512, 2>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
+                        if (p->Q == 16) launch_cluster(k_tree_pc<16, 512, 2>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
+                        else            launch_cluster(k_tree_pc<8, 512, 2>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
                     } else {
-                        if (p->Q == 16) launch_plain(k_tree_pc<16, 256, 4>, grid, 256, smem, s, a, (const float*)p->m2m, p->P, tabB);
-                        else            launch_plain(k_tree_pc<8, 256, 4>, grid, 256, smem, s, a, (const float*)p->m2m, p->P, tabB);
+                        if (p->Q == 16) launch_cluster(k_tree_pc<16, 256, 4>, grid, 256, smem, s, a, (const float*)p->m2m, p->P, tabB);
+                        else            launch_cluster(k_tree_pc<8, 256, 4>, grid, 256, smem, s, a, (const float*)p->m2m, p->P, tabB);
                     }
                     LAUNCH_CHECK();
                     continue;
@@ -979,6 +1005,22 @@ struct Exec {
         for (RankBufs& rb : p->ranks) {
             C* dst = out[p->virt ? rb.g : 0];
             const C* src = (const C*)(p->G > 1 ? rb.Rcv : rb.W);
+            if (p->row_cl) {                     // one pass per row on a cluster of row_cl CTAs
+                int in_row = (int)p->M, lblk = lM, blk_stride = 0;
+                if (p->G > 1) { in_row = (int)p->Mg; lblk = ilog2(p->Mg); blk_stride = (int)((p->P / p->G) * p->Mg); }
+                const int LKr = lM - ilog2(p->row_cl);
+                const size_t smem = ((size_t)(1 << LKr) + (1 << LKr) / 16 + p->M / 16 + 16 * p->row_cl) * sizeof(C);
+                const unsigned grid = (unsigned)(rows * p->row_cl);
+                dispatch<8, 9, 10, 11, 12, 13>(LKr, [&](auto lk) {
+                    constexpr int LK = decltype(lk)::value;
+                    if constexpr (LK <= kRowFftMax<R> - 1) {
+                        if (p->row_cl == 2) launch_cluster(k_fft_rowc<R, LK, 2>, grid, 1 << (LK - 4), smem, s, src, dst, (const C*)p->twM, in_row, lblk, blk_stride);
+                        else                launch_cluster(k_fft_rowc<R, LK, 4>, grid, 1 << (LK - 4), smem, s, src, dst, (const C*)p->twM, in_row, lblk, blk_stride);
+                    }
+                });
+                LAUNCH_CHECK();
+                continue;
+            }
             if (p->row_fft1) {                   // one pass per row, the row in shared memory
                 int in_row = (int)p->M, lblk = lM, blk_stride = 0;
                 if (p->G > 1) { in_row = (int)p->Mg; lblk = ilog2(p->Mg); blk_stride = (int)((p->P / p->G) * p->Mg); }
@@ -1214,6 +1256,14 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
         const int lM = ilog2(p->M);
         const char* e = getenv("FMMFFT_ROWFFT");
         p->row_fft1 = lM >= 8 && lM <= (precision == FMMFFT_C64 ? 14 : 13) && !(e && e[0] == '0');
+        // cluster rows (k_fft_rowc, FMMFFT_ROWFFT_CL=2|4): each row split over CL CTAs
+        const int kmax = precision == FMMFFT_C64 ? 13 : 12;
+        const long long rows = P / G;
+        int cl = 0;                      // measured slower than k_fft_row on cfg2 (opt-in)
+        (void)rows;
+        if (const char* c = getenv("FMMFFT_ROWFFT_CL")) cl = atoi(c);
+        if (cl == 4 && lM - 2 < 8) cl = 2;
+        if ((cl == 2 || cl == 4) && lM - ilog2(cl) >= 8 && lM - ilog2(cl) <= kmax && !(e && e[0] == '0')) p->row_cl = cl;
     }
     st = precision == FMMFFT_C64 ? build_tables<float>(p) : build_tables<double>(p);
     if (!st) {
@@ -1307,7 +1357,7 @@ fmmfft_status_t fmmfft_get_info(fmmfft_plan_t p, fmmfft_info_t* info) {
     info->L = p->L; info->precision = p->prec; info->M = p->M; info->level_gather = p->lg;
     info->n_stages = ST_COUNT + 1; info->workspace_bytes = p->ws_bytes; info->kernels_per_execute = p->kernels;
     info->variant = (p->tree_p ? FMMFFT_VARIANT_TREE_FUSED : 0u) | (p->s2t_tc ? FMMFFT_VARIANT_S2T_TC : 0u) |
-                    (p->row_fft1 ? FMMFFT_VARIANT_ROW_FFT1 : 0u);
+                    ((p->row_fft1 || p->row_cl) ? FMMFFT_VARIANT_ROW_FFT1 : 0u);
     return FMMFFT_SUCCESS;
 }
 

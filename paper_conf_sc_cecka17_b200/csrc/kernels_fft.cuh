@@ -9,6 +9,8 @@
 // transform length (template LLEN = log2 length): every stage's radix, shifts, masks and
 // twiddle strides are compile-time constants; 8 elements per thread per stage.
 #pragma once
+#include <cooperative_groups.h>
+
 #include "common.cuh"
 
 namespace fmmfft {
@@ -434,6 +436,123 @@ k_fft_row(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, const C2<R>* __
     if constexpr (L0 + 4 < LLEN) stage(std::integral_constant<int, L0 + 4>{});
     if constexpr (L0 + 8 < LLEN) stage(std::integral_constant<int, L0 + 8>{});
     static_assert(L0 + 12 >= LLEN, "k_fft_row: LLEN <= L0 + 12");
+}
+
+// ---------------------------------------------------------------------------------------------
+// k_fft_rowc: the M-point FFT of one row (§3 step 4) on a cluster of CL CTAs, M = CL K.
+// Four-step split m = m1 + CL m2, k = k2 + K k1 (m1, k1 < CL; m2, k2 < K):
+//     X[k2 + K k1] = sum_{m1} w_CL^{m1 k1} w_M^{m1 k2} [ sum_{m2} x[m1 + CL m2] w_K^{m2 k2} ].
+// CTA r: (1) loads the contiguous block x[r K, (r+1) K) (coalesced, through the all-to-all receive
+// layout like k_fft_pass); (2) gathers its decimated sequence x[r + CL m2] from the cluster's
+// blocks through distributed shared memory and runs the K-point Stockham FFT in shared memory
+// (radix R0 then radix 16, as k_fft_row; twiddles w_K^u = w_M^{CL u} from the same table),
+// multiplying the last stage's natural-order output by w_M^{r k2}; (3) takes k2 in
+// [r K/CL, (r+1) K/CL), reads the CL partial spectra of those k2 through DSMEM and finishes
+// with a radix-CL DFT, storing CL contiguous runs of the output row.
+// ---------------------------------------------------------------------------------------------
+template <int E, typename C> __device__ __forceinline__ void dft_small(C* v) {
+    if constexpr (E == 2) dft2(v);
+    else if constexpr (E == 4) dft4(v);
+    else if constexpr (E == 8) dft8(v);
+    else dft16(v);
+}
+
+template <typename R, int LK, int CL>
+__global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(1 << (LK - 4))
+k_fft_rowc(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, const C2<R>* __restrict__ twM,
+           int in_row, int lblk, int blk_stride) {
+    namespace cg = cooperative_groups;
+    using C = C2<R>;
+    constexpr int K = 1 << LK, NT = K >> 4;
+    constexpr int LCL = CL == 2 ? 1 : (CL == 4 ? 2 : 3);
+    constexpr int LM = LK + LCL, M = 1 << LM;
+    constexpr int L0 = (LK & 3) ? (LK & 3) : 4, R0 = 1 << L0, NB0 = 16 / R0;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    C* x = reinterpret_cast<C*>(smem_raw);                        // [row_pad(K)]
+    C* tw = x + row_pad(K);                                       // [M/16]  w_M^u
+    C* twc = tw + M / 16;                                         // [16 CL] w_{16 CL}^e
+    cg::cluster_group cluster = cg::this_cluster();
+    const int r = (int)cluster.block_rank();
+    const int tid = threadIdx.x;
+    const size_t row = blockIdx.x / CL;
+    for (int u = tid; u < M / 16; u += NT) cp_async_elem(tw + u, twM + u);
+    for (int e = tid; e < 16 * CL; e += NT) twc[e] = twiddle<R>(e, 16 * CL);
+    cp_async_commit();
+    pdl_wait();
+    // (1) contiguous block r of the row
+    {
+        const C* xin = in + row * (size_t)in_row;
+        const int bmask = (1 << lblk) - 1;
+        C v[16];
+#pragma unroll
+        for (int u = 0; u < 16; ++u) {
+            const int m = r * K + tid + u * NT;
+            v[u] = ldg_c(xin + (size_t)(m >> lblk) * blk_stride + (m & bmask));
+        }
+#pragma unroll
+        for (int u = 0; u < 16; ++u) x[row_pad(tid + u * NT)] = v[u];
+    }
+    cp_async_wait_all();
+    cluster.sync();
+    // (2) stage 0 of the K-point FFT on the decimated sequence y[m2] = x[r + CL m2] (DSMEM gather)
+    C v[16];
+#pragma unroll
+    for (int b = 0; b < NB0; ++b) {
+        const int j = tid + b * NT;
+#pragma unroll
+        for (int t = 0; t < R0; ++t) {
+            const int g = r + CL * (j + t * (K / R0));
+            v[b * R0 + t] = *cluster.map_shared_rank(x + row_pad(g & (K - 1)), g >> LK);
+        }
+    }
+#pragma unroll
+    for (int b = 0; b < NB0; ++b) dft_small<R0>(v + b * R0);
+    cluster.sync();                                              // every gather done: x is free
+#pragma unroll
+    for (int b = 0; b < NB0; ++b) {
+        const int j = tid + b * NT;
+#pragma unroll
+        for (int t = 0; t < R0; ++t) x[row_pad(j * R0 + t)] = v[b * R0 + t];
+    }
+    __syncthreads();
+    // radix-16 stages; the last one (Ns = K/16) gives Z[k2], k2 = j + t K/16, natural order
+    auto stage = [&](auto lnsc) {
+        constexpr int LNS = decltype(lnsc)::value, NS = 1 << LNS;
+        const int j = tid, k = j & (NS - 1);
+#pragma unroll
+        for (int t = 0; t < 16; ++t) v[t] = x[row_pad(j + t * NT)];
+        twiddle_powers<16>(v, tw[(k << (LK - 4 - LNS)) * CL]);  // w_K^u = w_M^{CL u}
+        dft16(v);
+        __syncthreads();
+        if constexpr (LNS + 4 < LK) {
+#pragma unroll
+            for (int t = 0; t < 16; ++t) x[row_pad(((j - k) << 4) + k + t * NS)] = v[t];
+        } else {                                                  // Z'[k2] = Z[k2] w_M^{r k2}
+            const C wj = tw[r * j];                               // w_M^{r j}, r j < M/16
+#pragma unroll
+            for (int t = 0; t < 16; ++t)                          // w_M^{r t K/16} = w_{16 CL}^{r t}
+                x[row_pad(j + t * NT)] = cmul(v[t], t ? cmul(wj, twc[(r * t) & (16 * CL - 1)]) : wj);
+        }
+        __syncthreads();
+    };
+    if constexpr (L0 < LK) stage(std::integral_constant<int, L0>{});
+    if constexpr (L0 + 4 < LK) stage(std::integral_constant<int, L0 + 4>{});
+    if constexpr (L0 + 8 < LK) stage(std::integral_constant<int, L0 + 8>{});
+    static_assert(L0 + 12 >= LK, "k_fft_rowc: LK <= L0 + 12");
+    cluster.sync();                                              // every partial spectrum written
+    // (3) k2 in [r K/CL, (r+1) K/CL): radix-CL DFT across the cluster's spectra
+    C* y = out + (row << LM);
+#pragma unroll
+    for (int u = 0; u < 16 / CL; ++u) {
+        const int k2 = r * (K / CL) + tid + u * NT;
+        C w[CL];
+#pragma unroll
+        for (int m1 = 0; m1 < CL; ++m1) w[m1] = *cluster.map_shared_rank(x + row_pad(k2), m1);
+        dft_small<CL>(w);
+#pragma unroll
+        for (int k1 = 0; k1 < CL; ++k1) y[k2 + K * k1] = w[k1];
+    }
+    cluster.sync();                                              // remote reads done before exit
 }
 
 }  // namespace fmmfft

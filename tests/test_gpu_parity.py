@@ -227,7 +227,9 @@ def test_full_size_sampled(F, N, P, B, Q, prec, G):
     {"FMMFFT_TREE_CL": "4"},     # far field on a cluster of 4 CTAs per FMM (k_tree_pc)
     {"FMMFFT_TREE": "w"},        # far field as wide per-level kernels (k_up, k_base, k_tree_down)
     {"FMMFFT_NO_GRAPH": "1"},    # eager launches instead of a CUDA graph
-    {"FMMFFT_ROWFFT": "0"},      # multi-pass M-point FFT (k_fft_pass) instead of k_fft_row
+    {"FMMFFT_ROWFFT": "0"},      # multi-pass M-point FFT (k_fft_pass) instead of k_fft_row(c)
+    {"FMMFFT_ROWFFT_CL": "0"},   # one CTA per M-point row (k_fft_row)
+    {"FMMFFT_ROWFFT_CL": "2"},   # a cluster of 2 CTAs per row (k_fft_rowc)
 ])
 @pytest.mark.parametrize("N,P,B,Q,G", [(1 << 20, 64, 2, 16, 1), (1 << 20, 64, 3, 16, 4)])
 def test_alternative_paths(F, monkeypatch, env, N, P, B, Q, G):
