@@ -209,6 +209,7 @@ struct fmmfft_plan_s {
     bool tree_p = false;             // use k_tree_p for the far field
     int tree_cl = 1;                 // k_tree_pc: CTAs per FMM (cluster), 1 = not used
     bool tree_phased = false;        // ... as up / all-levels M2L / L2L-chain launches (FMMFFT_TREE=p) (k_tree_pq<.., false>, k_m2l_flat, k_tree_dn)
+    bool lvl_off = false;            // FMMFFT_DOWN=tree: every down level in k_tree_down (no k_m2l_lvl)
     bool s2t_tc = false;             // S2T on tcgen05 (k_s2t_tc): complex64, M_L = 64, nb % 128 == 0
     void* toep = nullptr;            // its Toeplitz hi/lo operand table
     bool row_fft1 = false;           // M-point FFTs in one pass per row (k_fft_row), M fits smem
@@ -490,6 +491,9 @@ static fmmfft_status_t init_kernel_attrs() {
             set((const void*)k_tree_pc<8, 256, 4>);
         }
         if constexpr (sizeof(R) == 4) set((const void*)k_s2t_tc);
+        set((const void*)k_m2l_lvl<R, 8>);
+        set((const void*)k_m2l_lvl<R, 16>);
+        set((const void*)k_m2l_lvl<R, 24>);
         set((const void*)k_tree_p<R, 1>);
         set((const void*)k_tree_p<R, 2>);
         set((const void*)k_tree_p<R, 4>);
@@ -853,12 +857,13 @@ struct Exec {
         const int PC_ = p->PCd;
         const size_t smem = ((size_t)nbB + 1) * p->Q * PC_ * sizeof(C) + (size_t)p->Q * p->Q * PC_ * sizeof(R);
         if (ntg <= 32 && smem <= 200 * 1024) {
-            const int NTr = ntg <= 4 ? 4 : ntg <= 8 ? 8 : ntg <= 16 ? 16 : 32;
+            const int NTr = 4;                          // targets per CTA (grid y spans them)
+            const unsigned gy = (unsigned)((ntg + NTr - 1) / NTr);
             with_pcd([&](auto pc) {
                 constexpr int PCv = decltype(pc)::value;
-                dispatch<4, 8, 16, 32>(NTr, [&](auto ntv) {
+                dispatch<4>(NTr, [&](auto ntv) {
                     constexpr int NTv = decltype(ntv)::value;
-                    launch_pdl(k_base<R, NTv, PCv>, p->P / PCv, PCv * p->Q, smem, s, (const C*)rb.Mfull[p->B], outp, (C*)rb.r,
+                    launch_pdl(k_base<R, NTv, PCv>, dim3((unsigned)(p->P / PCv), gy), PCv * p->Q, smem, s, (const C*)rb.Mfull[p->B], outp, (C*)rb.r,
                                                                            (int)tgt_base, ntg, (const R*)p->m2lB,
                                                                            p->m2lB_chunk, nbB, p->P, p->Q);
                 });
@@ -896,57 +901,109 @@ struct Exec {
         return FMMFFT_SUCCESS;
     }
 
-    // ---- down: M2L + L2L for every level B+1 .. L in one launch per rank (k_tree_down)
+    // level l's source / output placement (global box indices -> buffers)
+    TreeLevel level_io(RankBufs& rb, int lev, long long g) const {
+        TreeLevel tl{};
+        const long long nbl = nb_at(lev);
+        tl.tab = p->m2l[lev];
+        if (p->G == 1) {
+            tl.src = interior(rb.Mpad[lev]); tl.src_base = 0; tl.src_mod = 1 << lev;
+            tl.out = rb.Lloc[lev]; tl.out_base = 0;
+        } else if (lev <= p->lg) {
+            tl.src = rb.Mfull[lev]; tl.src_base = 0; tl.src_mod = 1 << lev;
+            if (lev == p->lg) { tl.out = rb.Lloc[lev]; tl.out_base = g * nbl; }
+            else { tl.out = rb.Lfull[lev]; tl.out_base = 0; }
+        } else {
+            tl.src = rb.Mpad[lev]; tl.src_base = g * nbl - 2; tl.src_mod = 0;
+            tl.out = rb.Lloc[lev]; tl.out_base = g * nbl;
+        }
+        return tl;
+    }
+
+    // first level handled by the per-level kernel k_m2l_lvl (levels with >= 2 tiles per rank);
+    // the levels above it go to k_tree_down. FMMFFT_DOWN=tree keeps every level in k_tree_down.
+    int lvl_first() const {
+        if (p->lvl_off) return p->L + 1;
+        if (!(p->Q == 8 || p->Q == 16 || p->Q == 24)) return p->L + 1;
+        constexpr int PCl = lvl_pc<R>();
+        if (p->PCd % PCl || p->P % PCl) return p->L + 1;
+        for (int lev = std::max(p->B, p->lg) + 1; lev <= p->L; ++lev)
+            if (nb_at(lev) >= 2 * lvl_nt<R, 16>()) return lev;
+        return p->L + 1;
+    }
+
+    // ---- down: M2L + L2L for every level B+1 .. L: k_tree_down over the upper levels (one
+    // launch, per leaf range), then one k_m2l_lvl launch per wide level
     fmmfft_status_t down() {
         if (p->L == p->B || p->tree_p) return FMMFFT_SUCCESS;
+        const int lnew = lvl_first();
+        const int Lv = lnew - 1;                     // k_tree_down's (virtual) leaf level
         const int PC_ = p->PCd;
         const int npc = p->P / PC_;
         const int QPC = p->Q * PC_;
         int optin = 0;
         CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, p->device));
-        auto smem_of = [&](int nr, int db) {
-            return (size_t)(1 + db) * p->m2l_chunk * sizeof(R) + (size_t)(1 + db) * (nr + 6) * QPC * sizeof(C) +
-                   (size_t)nr * QPC * sizeof(C) + (size_t)(nr / 2 + 1) * QPC * sizeof(C) + (size_t)2 * p->Q * p->Q * sizeof(R);
-        };
-        int NR = std::min(16, p->nb);
-        while (NR > 1 && (long long)(p->nb / NR) * npc < 148) NR /= 2;
-        while (NR > 1 && smem_of(NR, 0) > (size_t)optin) NR /= 2;
-        const int db = smem_of(NR, 1) <= (size_t)optin ? 1 : 0;
-        const size_t smem = smem_of(NR, db);
         for (RankBufs& rb : p->ranks) {
             const long long g = grank(rb);
-            TreeDownArgs a{};
-            for (int lev = p->B + 1; lev <= p->L; ++lev) {
-                TreeLevel& tl = a.lev[lev];
-                const long long nbl = nb_at(lev);
-                tl.tab = p->m2l[lev];
-                if (p->G == 1) {
-                    tl.src = interior(rb.Mpad[lev]); tl.src_base = 0; tl.src_mod = 1 << lev;
-                    tl.out = rb.Lloc[lev]; tl.out_base = 0;
-                } else if (lev <= p->lg) {
-                    tl.src = rb.Mfull[lev]; tl.src_base = 0; tl.src_mod = 1 << lev;
-                    if (lev == p->lg) { tl.out = rb.Lloc[lev]; tl.out_base = g * nbl; }
-                    else { tl.out = rb.Lfull[lev]; tl.out_base = 0; }
-                } else {
-                    tl.src = rb.Mpad[lev]; tl.src_base = g * nbl - 2; tl.src_mod = 0;
-                    tl.out = rb.Lloc[lev]; tl.out_base = g * nbl;
-                }
-            }
-            if (p->lg == p->B) { a.par0 = rb.Lloc[p->B]; a.par0_base = g * nb_at(p->B); }
-            else { a.par0 = rb.Lfull[p->B]; a.par0_base = 0; }
-            a.leaf0 = g * p->nb;
-            a.lstart = p->B + 1;
-            a.L = p->L;
-            const dim3 grid((unsigned)(p->nb / NR), (unsigned)npc);
-            with_pcd([&](auto pc) {
-                constexpr int PCv = decltype(pc)::value;
-                dispatch<1, 2, 4, 8, 16>(NR, [&](auto nr) {
-                    constexpr int NRv = decltype(nr)::value;
-                    launch_pdl(k_tree_down<R, PCv, NRv>, grid, PCv * p->Q, smem, s, a, (const R*)p->m2m, p->P, p->Q,
-                                                                            p->m2l_chunk, db);
+            if (Lv > p->B) {
+                const int nbv = nb_at(Lv);
+                auto smem_of = [&](int nr, int db) {
+                    return (size_t)(1 + db) * p->m2l_chunk * sizeof(R) + (size_t)(1 + db) * (nr + 6) * QPC * sizeof(C) +
+                           (size_t)nr * QPC * sizeof(C) + (size_t)(nr / 2 + 1) * QPC * sizeof(C) + (size_t)2 * p->Q * p->Q * sizeof(R);
+                };
+                int NR = std::min(16, nbv);
+                while (NR > 1 && (long long)(nbv / NR) * npc < 148) NR /= 2;
+                while (NR > 1 && smem_of(NR, 0) > (size_t)optin) NR /= 2;
+                const int db = smem_of(NR, 1) <= (size_t)optin ? 1 : 0;
+                const size_t smem = smem_of(NR, db);
+                TreeDownArgs a{};
+                for (int lev = p->B + 1; lev <= Lv; ++lev) a.lev[lev] = level_io(rb, lev, g);
+                if (p->lg == p->B) { a.par0 = rb.Lloc[p->B]; a.par0_base = g * nb_at(p->B); }
+                else { a.par0 = rb.Lfull[p->B]; a.par0_base = 0; }
+                a.leaf0 = g * nbv;
+                a.lstart = p->B + 1;
+                a.L = Lv;
+                const dim3 grid((unsigned)(nbv / NR), (unsigned)npc);
+                with_pcd([&](auto pc) {
+                    constexpr int PCv = decltype(pc)::value;
+                    dispatch<1, 2, 4, 8, 16>(NR, [&](auto nr) {
+                        constexpr int NRv = decltype(nr)::value;
+                        launch_pdl(k_tree_down<R, PCv, NRv>, grid, PCv * p->Q, smem, s, a, (const R*)p->m2m, p->P, p->Q,
+                                                                                p->m2l_chunk, db);
+                    });
                 });
-            });
-            LAUNCH_CHECK();
+                LAUNCH_CHECK();
+            }
+            for (int lev = lnew; lev <= p->L; ++lev) {
+                const TreeLevel tl = level_io(rb, lev, g);
+                LvlArgs la{};
+                la.src = tl.src; la.src_base = tl.src_base; la.src_mod = tl.src_mod;
+                la.out = tl.out; la.out_base = tl.out_base;
+                if (lev - 1 == p->B) {
+                    if (p->lg == p->B) { la.par = rb.Lloc[p->B]; la.par_base = g * nb_at(p->B); }
+                    else { la.par = rb.Lfull[p->B]; la.par_base = 0; }
+                } else {
+                    const TreeLevel tp = level_io(rb, lev - 1, g);
+                    la.par = tp.out; la.par_base = tp.out_base;
+                }
+                la.tab = tl.tab; la.tab_chunk = p->m2l_chunk; la.PCd = p->PCd;
+                la.tgt0 = g * nb_at(lev);
+                constexpr int PCl = lvl_pc<R>();
+                const int nsub = p->P / PCl;
+                bool ok = dispatch<8, 16, 24>(p->Q, [&](auto qv) {
+                    constexpr int QV = decltype(qv)::value;
+                    constexpr int NT = lvl_nt<R, QV>();
+                    la.ntiles = nb_at(lev) / NT;
+                    const size_t smem = lvl_smem<R, QV>();
+                    const int per_sm = std::max(1, std::min(2, (int)((size_t)(optin + 1024) / (smem + 1024))));
+                    const int target = 148 * per_sm;
+                    const int nseg = (int)std::max(1LL, std::min<long long>(la.ntiles, (target + nsub - 1) / nsub));
+                    launch_pdl(k_m2l_lvl<R, QV>, dim3((unsigned)nseg, (unsigned)nsub), lvl_threads<R, QV>(), smem, s, la,
+                               (const R*)p->m2m, p->P);
+                });
+                if (!ok) return fail(FMMFFT_UNSUPPORTED, "k_m2l_lvl: Q=%d", p->Q);
+                LAUNCH_CHECK();
+            }
         }
         return FMMFFT_SUCCESS;
     }
@@ -1249,6 +1306,7 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
     // tiles per rank; FMMFFT_S2T=simt selects the FFMA2 kernel (k_near_up) instead
     p->s2t_tc = precision == FMMFFT_C64 && M_L == 64 && (p->nb % S2TC_BOXES) == 0;
     if (const char* e = getenv("FMMFFT_S2T")) p->s2t_tc = p->s2t_tc && e[0] == 't';
+    if (const char* e = getenv("FMMFFT_DOWN")) p->lvl_off = e[0] == 't';
     const char* g_env = getenv("FMMFFT_NO_GRAPH");
     p->use_graph = !(g_env && g_env[0] == '1');
     plan_radices(p);

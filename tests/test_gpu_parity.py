@@ -65,6 +65,9 @@ def rel(a, b):
     (1 << 17, 2, 3, 16, "c64", 128),       # P = 2, M_L = 128
     (1 << 19, 512, 2, 16, "c64", 16),      # P = 512 (cfg4's P/G shape)
     (1 << 16, 4, 5, 16, "c64", 32),
+    (1 << 20, 16, 4, 16, "c64", 64),       # wide tree (L = 10): per-level k_m2l_lvl for l >= 6
+    (1 << 20, 16, 4, 24, "c128", 16),      # L = 12, Q = 24, fp64 k_m2l_lvl
+    (1 << 20, 32, 3, 8, "c64", 32),        # L = 10, Q = 8
 ])
 def test_end_to_end_vs_dft(F, N, P, B, Q, prec, M_L):
     plan, x, y = run(F, N, P, B, Q, prec, M_L)
@@ -121,6 +124,8 @@ def test_stages_match_oracle(F, prec, N, P, B, Q, M_L):
     (1 << 16, 16, 2, 16, "c128", 64, 8),     # L = 6, l_g = 4
     (1 << 15, 16, 2, 16, "c64", 64, 8),      # L = 5: one box per rank at level 3
     (1 << 20, 128, 2, 24, "c128", 64, 8),    # cfg4 shape, reduced N
+    (1 << 20, 32, 2, 16, "c64", 32, 4),      # 256 leaves per rank: k_m2l_lvl on halo'd levels 8..10
+    (1 << 20, 16, 3, 16, "c128", 16, 2),     # fp64 k_m2l_lvl, 2048 leaves per rank
 ])
 def test_virtual_ranks_vs_oracle(F, N, P, B, Q, prec, M_L, G):
     plan, x, y = run(F, N, P, B, Q, prec, M_L, G=G, virtual=True)
@@ -225,7 +230,8 @@ def test_full_size_sampled(F, N, P, B, Q, prec, G):
     {"FMMFFT_S2T": "simt"},      # S2T on the FFMA2 SIMT kernel (k_near_up) instead of tcgen05
     {"FMMFFT_TREE": "f"},        # far field fused in one per-FMM kernel (k_tree_pq)
     {"FMMFFT_TREE_CL": "4"},     # far field on a cluster of 4 CTAs per FMM (k_tree_pc)
-    {"FMMFFT_TREE": "w"},        # far field as wide per-level kernels (k_up, k_base, k_tree_down)
+    {"FMMFFT_TREE": "w"},        # far field as wide per-level kernels (k_up, k_base, k_tree_down + k_m2l_lvl)
+    {"FMMFFT_TREE": "w", "FMMFFT_DOWN": "tree"},   # ... with every down level in k_tree_down
     {"FMMFFT_NO_GRAPH": "1"},    # eager launches instead of a CUDA graph
     {"FMMFFT_ROWFFT": "0"},      # multi-pass M-point FFT (k_fft_pass) instead of k_fft_row(c)
     {"FMMFFT_ROWFFT_CL": "0"},   # one CTA per M-point row (k_fft_row)
