@@ -209,6 +209,7 @@ struct fmmfft_plan_s {
     bool tree_p = false;             // use k_tree_p for the far field
     int tree_cl = 1;                 // k_tree_pc: CTAs per FMM (cluster), 1 = not used
     bool tree_phased = false;        // ... as up / all-levels M2L / L2L-chain launches (FMMFFT_TREE=p) (k_tree_pq<.., false>, k_m2l_flat, k_tree_dn)
+    int fs_lc1 = 0, fs_lc2 = 0, fs_lr = 0;   // four-step large-M FFT: column pass bits (2nd: 0 = none), row pass bits
     bool lvl_off = false;            // FMMFFT_DOWN=tree: every down level in k_tree_down (no k_m2l_lvl)
     bool s2t_tc = false;             // S2T on tcgen05 (k_s2t_tc): complex64, M_L = 64, nb % 128 == 0
     void* toep = nullptr;            // its Toeplitz hi/lo operand table
@@ -377,6 +378,9 @@ static fmmfft_status_t build_tables(fmmfft_plan_s* p) {
 
 static constexpr int kTileF = 8192, kTileD = 4096;   // shared FFT tile (elements)
 template <typename R> static constexpr int kRowFftMax = sizeof(R) == 4 ? 14 : 13;   // k_fft_row: whole row in smem
+// four-step passes: largest pass length (log2) and columns (rows) per CTA for a pass of 2^l points
+template <typename R> __host__ __device__ constexpr int fs_max() { return sizeof(R) == 4 ? 11 : 10; }
+template <typename R> __host__ __device__ constexpr int fs_cols(int l) { return l <= fs_max<R>() - 1 ? 16 : 8; }
 
 static void plan_radices(fmmfft_plan_s* p) {
     const int maxbits = p->prec == FMMFFT_C64 ? 10 : 9;
@@ -513,6 +517,14 @@ static fmmfft_status_t init_kernel_attrs() {
                 if constexpr (LK <= kRowFftMax<R> - 1) {
                     set((const void*)k_fft_rowc<R, LK, 2>);
                     set((const void*)k_fft_rowc<R, LK, 4>);
+                }
+            });
+        for (int l = 5; l <= fs_max<R>(); ++l)
+            dispatch<5, 6, 7, 8, 9, 10, 11>(l, [&](auto v) {
+                constexpr int LV = decltype(v)::value;
+                if constexpr (LV <= fs_max<R>()) {
+                    set((const void*)k_fft_col<R, LV, fs_cols<R>(LV)>);
+                    set((const void*)k_fft_rowt<R, LV, fs_cols<R>(LV)>);
                 }
             });
         for (int ll = 8; ll <= kRowFftMax<R>; ++ll)
@@ -1054,14 +1066,57 @@ struct Exec {
         return FMMFFT_SUCCESS;
     }
 
+    // one column pass of the four-step M-FFT (k_fft_col): nseq sequences of length 2^lMs
+    fmmfft_status_t col_pass(const C* in_, C* out_, int LCv, int lMs, int lSdiv, long long in_row, int lblk,
+                             long long blk_stride, long long nseq) {
+        const int lMi = lMs - LCv;
+        bool ok = dispatch<5, 6, 7, 8, 9, 10, 11>(LCv, [&](auto lc) {
+            constexpr int LC = decltype(lc)::value;
+            constexpr int CB = fs_cols<R>(LC);
+            if constexpr (LC <= fs_max<R>())
+                launch_pdl(k_fft_col<R, LC, CB>, dim3((unsigned)((1LL << lMi) / CB), (unsigned)nseq), CB << (LC - 4),
+                           fft_col_smem<R, LC, CB>(), s, in_, out_, lMs, lMi, lSdiv, (long long)p->M, in_row, lblk, blk_stride);
+        });
+        if (!ok) return fail(FMMFFT_UNSUPPORTED, "k_fft_col: 2^%d", LCv);
+        LAUNCH_CHECK();
+        return FMMFFT_SUCCESS;
+    }
+
     // ---- M-point FFTs over the P/G local rows
     fmmfft_status_t mfft() {
+        fmmfft_status_t st_;
         const int n = (int)p->radices.size();
         const long long rows = p->P / p->G;
         const int lM = ilog2(p->M);
         for (RankBufs& rb : p->ranks) {
             C* dst = out[p->virt ? rb.g : 0];
             const C* src = (const C*)(p->G > 1 ? rb.Rcv : rb.W);
+            if (p->fs_lr) {                      // four-step: column pass(es) + transposing row pass
+                long long in_row = p->M, blk_stride = 0;
+                int lblk = 62;
+                if (p->G > 1) { in_row = p->Mg; lblk = ilog2(p->Mg); blk_stride = (p->P / p->G) * p->Mg; }
+                const int npass = p->fs_lc2 ? 3 : 2;
+                C* a1out = npass == 3 ? dst : (C*)rb.tmp;
+                if ((st_ = col_pass(src, a1out, p->fs_lc1, lM, 0, in_row, lblk, blk_stride, rows))) return st_;
+                const C* bsrc = a1out;
+                if (npass == 3) {
+                    const int lMs = lM - p->fs_lc1;
+                    if ((st_ = col_pass(dst, (C*)rb.tmp, p->fs_lc2, lMs, p->fs_lc1, 1LL << lMs, 62, 0, rows << p->fs_lc1))) return st_;
+                    bsrc = (const C*)rb.tmp;
+                }
+                const int lrpr = lM - p->fs_lr;
+                const long long trows = rows << lrpr;
+                bool ok = dispatch<5, 6, 7, 8, 9, 10, 11>(p->fs_lr, [&](auto ll) {
+                    constexpr int LL = decltype(ll)::value;
+                    constexpr int CR = fs_cols<R>(LL);
+                    if constexpr (LL <= fs_max<R>())
+                        launch_pdl(k_fft_rowt<R, LL, CR>, (unsigned)(trows / CR), CR << (LL - 4), fft_rowt_smem<R, LL, CR>(), s,
+                                   bsrc, dst, (long long)p->M, lrpr);
+                });
+                if (!ok) return fail(FMMFFT_UNSUPPORTED, "k_fft_rowt: 2^%d", p->fs_lr);
+                LAUNCH_CHECK();
+                continue;
+            }
             if (p->row_cl) {                     // one pass per row on a cluster of row_cl CTAs
                 int in_row = (int)p->M, lblk = lM, blk_stride = 0;
                 if (p->G > 1) { in_row = (int)p->Mg; lblk = ilog2(p->Mg); blk_stride = (int)((p->P / p->G) * p->Mg); }
@@ -1322,6 +1377,23 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
         if (const char* c = getenv("FMMFFT_ROWFFT_CL")) cl = atoi(c);
         if (cl == 4 && lM - 2 < 8) cl = 2;
         if ((cl == 2 || cl == 4) && lM - ilog2(cl) >= 8 && lM - ilog2(cl) <= kmax && !(e && e[0] == '0')) p->row_cl = cl;
+    }
+    {   // rows longer than one CTA's shared memory: the four-step passes (FMMFFT_MFFT=pass keeps k_fft_pass)
+        const int lM = ilog2(p->M);
+        const int mx = precision == FMMFFT_C64 ? 11 : 10;
+        const char* e = getenv("FMMFFT_MFFT");
+        const bool want = !(e && e[0] == 'p') && !(getenv("FMMFFT_ROWFFT") && getenv("FMMFFT_ROWFFT")[0] == '0');
+        if (want && !p->row_fft1 && !p->row_cl && lM >= 10 && lM <= 3 * mx) {
+            if (lM <= 2 * mx) {
+                p->fs_lr = std::min(mx, (lM + 1) / 2);
+                p->fs_lc1 = lM - p->fs_lr;
+            } else {
+                p->fs_lr = std::min(mx, (lM + 2) / 3);
+                p->fs_lc1 = std::min(mx, (lM - p->fs_lr + 1) / 2);
+                p->fs_lc2 = lM - p->fs_lr - p->fs_lc1;
+            }
+            if (p->fs_lc1 < 5 || p->fs_lr < 5 || (p->fs_lc2 && p->fs_lc2 < 5)) p->fs_lr = p->fs_lc1 = p->fs_lc2 = 0;
+        }
     }
     st = precision == FMMFFT_C64 ? build_tables<float>(p) : build_tables<double>(p);
     if (!st) {

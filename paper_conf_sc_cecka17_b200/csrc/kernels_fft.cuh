@@ -555,4 +555,155 @@ k_fft_rowc(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, const C2<R>* _
     cluster.sync();                                              // remote reads done before exit
 }
 
+
+// ---------------------------------------------------------------------------------------------
+// Large M (rows that do not fit one CTA's shared memory): the M-point FFT (§3 step 4) as a
+// four-step split over 2 or 3 passes, each pass reading and writing HBM once with >= 64-byte runs.
+// For M = M1 M2 (M3): n = n1 M2 M3 + n2 M3 + n3, k = k1 + M1 k2 + M1 M2 k3,
+//   X[k] = sum_{n3} w_{M3}^{n3 k3} w_{M2 M3}^{n3 k2} sum_{n2} w_{M2}^{n2 k2} w_M^{n2' k1} sum_{n1} w_{M1}^{n1 k1} x[n],
+// with n2' = n2 M3 + n3 the inner index of the first pass. A column pass (k_fft_col) takes
+// sequences of length Ms = Mc Mi, FFTs the Mc-point columns (stride Mi) of CB adjacent inner
+// indices at once and multiplies by w_{Ms}^{n_inner k_col}; the row pass (k_fft_rowt) FFTs CR
+// contiguous rows of length Mr and stores them transposed, X[k_prefix + (M / Mr) k_last], CR
+// consecutive prefixes at a time. Both use k_fft_row's scheme (radix R0 then radix-16 stages,
+// 16 elements per thread, one pad element per 16) on CB (CR) columns side by side; the column
+// stride CS = 16/CB (mod 16) makes the column-parallel accesses conflict-free.
+// ---------------------------------------------------------------------------------------------
+template <int LEN, int NCOL> __host__ __device__ constexpr int col_stride() {
+    return ((row_pad(LEN) + 15) / 16) * 16 + 16 / NCOL;
+}
+template <typename R, int LC, int CB> __host__ __device__ constexpr size_t fft_col_smem() {
+    return ((size_t)CB * col_stride<1 << LC, CB>() + ((1 << LC) >> 4)) * sizeof(C2<R>);
+}
+
+// radix-16 stage LNS (Ns = 2^LNS) of a 2^LL-point Stockham FFT on column xc, thread j of NT;
+// the caller handles the last stage (LNS + 4 == LL)
+template <int LL, int LNS, typename C>
+__device__ __forceinline__ void row_stage_mid(C* xc, const C* tw, int j, C* v) {
+    constexpr int NT = (1 << LL) >> 4, NS = 1 << LNS;
+    const int k = j & (NS - 1);
+#pragma unroll
+    for (int t = 0; t < 16; ++t) v[t] = xc[row_pad(j + t * NT)];
+    twiddle_powers<16>(v, tw[k << (LL - 4 - LNS)]);
+    dft16(v);
+    __syncthreads();
+#pragma unroll
+    for (int t = 0; t < 16; ++t) xc[row_pad(((j - k) << 4) + k + t * NS)] = v[t];
+    __syncthreads();
+}
+
+template <typename R, int LC, int CB>
+__global__ void __launch_bounds__(CB << (LC - 4))
+k_fft_col(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, int lMs, int lMi, int lSdiv, long long M,
+          long long in_row, int lblk, long long blk_stride) {
+    pdl_trigger();
+    using C = C2<R>;
+    constexpr int Mc = 1 << LC, NT = Mc >> 4, CS = col_stride<Mc, CB>();
+    constexpr int L0 = (LC & 3) ? (LC & 3) : 4, R0 = 1 << L0, NB0 = 16 / R0;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    C* x = reinterpret_cast<C*>(smem_raw);                        // [CB][CS]
+    C* tw = x + CB * CS;                                          // [Mc/16]  w_Mc^u
+    const int tid = threadIdx.x, c = tid % CB, j = tid / CB;
+    for (int u = tid; u < NT; u += blockDim.x) tw[u] = twiddle_pow2(R(0), u, LC);
+    const long long s = blockIdx.y;
+    const long long n2 = (long long)blockIdx.x * CB + c;          // inner index of this column
+    const long long Mi = 1LL << lMi;
+    const long long bmask = (1LL << lblk) - 1;
+    const C* xin = in + s * in_row;
+    C* xc = x + c * CS;
+    pdl_wait();
+    C v[16];
+#pragma unroll
+    for (int b = 0; b < NB0; ++b) {
+        const int jj = j + b * NT;
+#pragma unroll
+        for (int t = 0; t < R0; ++t) {
+            const long long m = (long long)(jj + t * (Mc / R0)) * Mi + n2;
+            v[b * R0 + t] = ldg_c(xin + (m >> lblk) * blk_stride + (m & bmask));
+        }
+    }
+#pragma unroll
+    for (int b = 0; b < NB0; ++b) dftR<R0>(v + b * R0);
+#pragma unroll
+    for (int b = 0; b < NB0; ++b) {
+        const int jj = j + b * NT;
+#pragma unroll
+        for (int t = 0; t < R0; ++t) xc[row_pad(jj * R0 + t)] = v[b * R0 + t];
+    }
+    __syncthreads();
+    if constexpr (L0 + 4 < LC) row_stage_mid<LC, L0>(xc, tw, j, v);
+    if constexpr (L0 + 8 < LC) row_stage_mid<LC, L0 + 4>(xc, tw, j, v);
+    static_assert(L0 + 12 >= LC, "k_fft_col: LC <= L0 + 12");
+    // last stage (Ns = Mc/16, k = j): natural order k_col = j + t NT, times w_Ms^{n2 k_col}
+    constexpr int LNS = LC - 4;
+#pragma unroll
+    for (int t = 0; t < 16; ++t) v[t] = xc[row_pad(j + t * NT)];
+    if constexpr (LNS > 0) twiddle_powers<16>(v, tw[j]);
+    dft16(v);
+    const long long Ms_mask = (1LL << lMs) - 1;
+    const C wb = twiddle_pow2(R(0), (int)((n2 * j) & Ms_mask), lMs);
+    twiddle_powers<16>(v, twiddle_pow2(R(0), (int)((n2 * NT) & Ms_mask), lMs));
+    const long long hi = s >> lSdiv, lo = s & ((1LL << lSdiv) - 1);
+    const long long kstride = Mi << lSdiv;
+    C* y = out + hi * M + lo * Mi + n2;
+#pragma unroll
+    for (int t = 0; t < 16; ++t) y[(long long)(j + t * NT) * kstride] = cmul(v[t], wb);
+}
+
+template <typename R, int LL, int CR> __host__ __device__ constexpr size_t fft_rowt_smem() {
+    return ((size_t)CR * col_stride<1 << LL, CR>() + ((1 << LL) >> 4)) * sizeof(C2<R>);
+}
+
+template <typename R, int LL, int CR>
+__global__ void __launch_bounds__(CR << (LL - 4))
+k_fft_rowt(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, long long M, int lrpr) {
+    pdl_trigger();
+    using C = C2<R>;
+    constexpr int Mr = 1 << LL, NT = Mr >> 4, CS = col_stride<Mr, CR>();
+    constexpr int L0 = (LL & 3) ? (LL & 3) : 4, R0 = 1 << L0, NB0 = 16 / R0;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    C* x = reinterpret_cast<C*>(smem_raw);                        // [CR][CS]
+    C* tw = x + CR * CS;                                          // [Mr/16]  w_Mr^u
+    const int tid = threadIdx.x;
+    for (int u = tid; u < NT; u += blockDim.x) tw[u] = twiddle_pow2(R(0), u, LL);
+    const long long r0 = (long long)blockIdx.x * CR;              // first row (global)
+    // stages 0 .. last-1: j fastest (row r = tid / NT), coalesced row loads
+    const int jr = tid % NT, rr = tid / NT;
+    C* xr = x + rr * CS;
+    pdl_wait();
+    C v[16];
+    const C* xin = in + ((r0 + rr) << LL);
+#pragma unroll
+    for (int b = 0; b < NB0; ++b) {
+        const int jj = jr + b * NT;
+#pragma unroll
+        for (int t = 0; t < R0; ++t) v[b * R0 + t] = ldg_c(xin + jj + t * (Mr / R0));
+    }
+#pragma unroll
+    for (int b = 0; b < NB0; ++b) dftR<R0>(v + b * R0);
+#pragma unroll
+    for (int b = 0; b < NB0; ++b) {
+        const int jj = jr + b * NT;
+#pragma unroll
+        for (int t = 0; t < R0; ++t) xr[row_pad(jj * R0 + t)] = v[b * R0 + t];
+    }
+    __syncthreads();
+    if constexpr (L0 + 4 < LL) row_stage_mid<LL, L0>(xr, tw, jr, v);
+    if constexpr (L0 + 8 < LL) row_stage_mid<LL, L0 + 4>(xr, tw, jr, v);
+    static_assert(L0 + 12 >= LL, "k_fft_rowt: LL <= L0 + 12");
+    // last stage: row fastest (r = tid % CR), stores of CR consecutive outputs per k
+    constexpr int LNS = LL - 4;
+    const int r = tid % CR, j = tid / CR;
+    const C* xc = x + r * CS;
+#pragma unroll
+    for (int t = 0; t < 16; ++t) v[t] = xc[row_pad(j + t * NT)];
+    if constexpr (LNS > 0) twiddle_powers<16>(v, tw[j]);
+    dft16(v);
+    const long long rg = r0 + r;
+    const long long row = rg >> lrpr, pre = rg & ((1LL << lrpr) - 1);
+    C* y = out + row * M + pre;
+#pragma unroll
+    for (int t = 0; t < 16; ++t) y[(long long)(j + t * NT) << lrpr] = v[t];
+}
+
 }  // namespace fmmfft

@@ -14,6 +14,8 @@ def load(path):
             continue
         if hdr and len(r) == len(hdr):
             d = dict(zip(hdr, r))
+            if d.get("Metric Name", "gpu__time_duration.sum") != "gpu__time_duration.sum":
+                continue
             name = d["Kernel Name"].split("(")[0].replace("void ", "")
             out.append((name, d["Grid Size"], d["Block Size"], float(d["Metric Value"])))
     return out

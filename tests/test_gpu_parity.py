@@ -252,3 +252,19 @@ def test_alternative_paths(F, monkeypatch, env, N, P, B, Q, G):
         assert np.array_equal(Tn[:, :, 0], x.reshape(2 ** L, 64, P)[:, :, 0])
         LL = plan.debug_buffer("L", L).cpu().numpy().reshape(2 ** L, Q, P)
         assert rel(LL[:, :, 1:], st["L"][L]) < TOL_STAGE[prec]
+
+
+# ------------------------------------------------------------------ large-M four-step FFT passes
+@pytest.mark.parametrize("N,P,prec,G,env", [
+    (1 << 23, 2, "c64", 1, None),        # M = 2^22: column pass 2^11 + transposing row pass 2^11
+    (1 << 24, 2, "c64", 1, None),        # M = 2^23: two column passes + row pass
+    (1 << 22, 2, "c128", 1, None),       # fp64, M = 2^21: three passes of 2^7
+    (1 << 21, 4, "c128", 1, None),       # fp64, M = 2^19: 2^9 + 2^10
+    (1 << 23, 4, "c64", 4, None),        # first column pass reads the all-to-all receive layout
+    (1 << 21, 4, "c64", 1, {"FMMFFT_MFFT": "pass"}),   # the multi-pass Stockham kernel instead
+])
+def test_large_m_fft(F, monkeypatch, N, P, prec, G, env):
+    for k, v in (env or {}).items():
+        monkeypatch.setenv(k, v)
+    plan, x, y = run(F, N, P, 2, 16, prec, 64, G=G, virtual=G > 1)
+    assert rel(y, O.fft_radix2(x)) < TOL_E2E[prec]
