@@ -466,7 +466,8 @@ static fmmfft_status_t init_kernel_attrs() {
         auto per_pc = [&](auto pc) {
             constexpr int PCv = decltype(pc)::value;
             set((const void*)k_near_up<R, IB, PCv>);
-            set((const void*)k_s2m<R, PCv>);
+            for (int lml = 4; lml <= 7; ++lml)
+                dispatch<4, 5, 6, 7>(lml, [&](auto v) { set((const void*)k_s2m<R, PCv, decltype(v)::value>); });
             if constexpr (PCv <= (sizeof(R) == 4 ? 16 : 8)) {
                 set((const void*)k_up<R, PCv>);
                 set((const void*)k_m2l_flat<R, 8, PCv>);
@@ -496,6 +497,9 @@ static fmmfft_status_t init_kernel_attrs() {
         }
         if constexpr (sizeof(R) == 4) set((const void*)k_s2t_tc);
         set((const void*)k_m2l_lvl<R, 8>);
+        set((const void*)k_m2m_lvl<R, 8>);
+        set((const void*)k_m2m_lvl<R, 16>);
+        set((const void*)k_m2m_lvl<R, 24>);
         set((const void*)k_m2l_lvl<R, 16>);
         set((const void*)k_m2l_lvl<R, 24>);
         set((const void*)k_tree_p<R, 1>);
@@ -634,8 +638,10 @@ struct Exec {
             dispatch<2, 4, 8, 16, 32>(PCs, [&](auto pc) {
                 constexpr int PCv = decltype(pc)::value;
                 if constexpr (!(sizeof(R) == 8 && PCv > 16))
-                    launch_pdl(k_s2m<R, PCv>, grid, PCv * (Qp / 4) * nbx, smem, s, S, interior(rb.Mpad[p->L]), (const R*)p->s2mT, p->P,
-                                                                           p->M_L, p->Q, (C*)rb.Sp, (C*)rb.Tn, p->nb, nbx);
+                    dispatch<4, 5, 6, 7>(ilog2(p->M_L), [&](auto lml) {
+                        launch_pdl(k_s2m<R, PCv, decltype(lml)::value>, grid, PCv * (Qp / 4) * nbx, smem, s, S, interior(rb.Mpad[p->L]),
+                                   (const R*)p->s2mT, p->P, p->Q, (C*)rb.Sp, (C*)rb.Tn, p->nb, nbx);
+                    });
             });
             LAUNCH_CHECK();
         }
@@ -705,6 +711,28 @@ struct Exec {
         int cur = from;
         const C* src = inl;
         long long nbc = nb_from;
+        // wide levels: one register-blocked k_m2m_lvl launch per level (>= 2 tiles of parents)
+        constexpr int PCl = lvl_pc<R>();
+        const bool lvl_ok = !p->lvl_off && (p->Q == 8 || p->Q == 16 || p->Q == 24) && p->PCd % PCl == 0 && p->P % PCl == 0;
+        int optin = 0;
+        CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, p->device));
+        while (lvl_ok && cur > to && (nbc >> 1) >= 2 * lvl_nt<R, 16>()) {
+            C* o = (C*)outs(cur - 1);
+            const int nsub = p->P / PCl;
+            dispatch<8, 16, 24>(p->Q, [&](auto qv) {
+                constexpr int QV = decltype(qv)::value;
+                const int ntiles = (int)((nbc >> 1) / lvl_nt<R, QV>());
+                const size_t smem = m2m_lvl_smem<R, QV>();
+                const int per_sm = std::max(1, std::min(2, (int)((size_t)(optin + 1024) / (smem + 1024))));
+                const int nseg = (int)std::max(1LL, std::min<long long>(ntiles, (148LL * per_sm + nsub - 1) / nsub));
+                launch_pdl(k_m2m_lvl<R, QV>, dim3((unsigned)nseg, (unsigned)nsub), lvl_threads<R, QV>(), smem, s, src, o,
+                           (const R*)p->m2m, p->P, ntiles);
+            });
+            LAUNCH_CHECK();
+            src = o;
+            nbc >>= 1;
+            --cur;
+        }
         while (cur > to) {
             int h = std::min(4, cur - to);
             while ((1LL << h) > nbc) --h;
