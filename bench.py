@@ -120,7 +120,7 @@ def load_traffic(workload: str, G: int, kernel: str):
         return None
 
 
-def stage_rooflines(N, P, B, Q, M_L, G, L, prec, tree_fused):
+def stage_rooflines(N, P, B, Q, M_L, G, L, prec, tree_fused, s2t_tc, mfft_kernel):
     """Algorithmic work per launch of each kernel stage, restated from PAPER.md §5.1:
     complex x real multiply-adds cost 2C = 4 real flops; the FFT stages are HBM-bound and move
     their input and output once. Returns {stage: (kernel, bound, amount)}."""
@@ -129,16 +129,42 @@ def stage_rooflines(N, P, B, Q, M_L, G, L, prec, tree_fused):
     esz = 8 if prec == "c64" else 16
     up = sum(2 ** l for l in range(B, L)) / G                      # parents formed by M2M
     dn = sum(2 ** l for l in range(B + 1, L + 1)) / G              # targets of M2L / L2L
-    tree = 2 * C * fmm * Q * Q * (2 * up + 3 * dn + dn) + 2 * C * fmm * Q * Q * 2 ** B * (2 ** B - 3) / G
+    m2m = 2 * C * fmm * Q * Q * 2 * up
+    down = 2 * C * fmm * Q * Q * 4 * dn
+    base = 2 * C * fmm * Q * Q * 2 ** B * (2 ** B - 3) / G
     out = {
         "s2m": ("k_s2m", "alu", 2 * C * M_L * nb * fmm * Q),
-        "s2t": ("k_near_up", "alu", 6 * C * M_L * M_L * nb * fmm),
+        "s2t": (("k_s2t_tc", "tensor") if s2t_tc else ("k_near_up", "alu")) + (6 * C * M_L * M_L * nb * fmm,),
         "post_pfft": ("k_post_pfft", "hbm", (N // G) * esz * 2 + nb * Q * P * esz),
-        "mfft": ("k_fft_pass / k_fft_row", "hbm", (N // G) * esz * 2),
+        "mfft": (mfft_kernel, "hbm", (N // G) * esz * 2),
     }
     if tree_fused:
-        out["top"] = ("k_tree_pq", "alu", tree)
+        out["top"] = ("k_tree_pc / k_tree_pq", "alu", m2m + down + base)
+    else:
+        out["m2m"] = ("k_m2m_lvl + k_up", "alu", m2m)
+        out["top"] = ("k_base", "alu", base)
+        out["down"] = ("k_m2l_lvl + k_tree_down", "alu", down)
     return out
+
+
+def cufft_comparator(x, flush, steps):
+    """cuFFT (torch.fft.fft, the library 1D FFT) on the same device, input, L2 flush and event
+    timing as the timed loop: the single-GPU comparator of BASELINE.json's "speedup vs cuFFTXt".
+    A library call for context, not part of the product path."""
+    import torch
+    for _ in range(3):
+        torch.fft.fft(x)
+    torch.cuda.synchronize()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    for a, b_ in ev:
+        flush.zero_()
+        a.record()
+        torch.fft.fft(x)
+        b_.record()
+    torch.cuda.synchronize()
+    ms = sum(a.elapsed_time(b_) for a, b_ in ev) / steps
+    return {"lib": "cuFFT via torch.fft.fft (1 GPU)", "value": flops_fft(x.numel()) / (ms * 1e-3) / 1e9,
+            "unit": "GFLOP/s", "ms_per_step": ms}
 
 
 # ------------------------------------------------------------------------------ CPU oracle legs
@@ -345,6 +371,7 @@ def run_fmmfft(args, rank, world, local_rank):
         dist.all_reduce(nx)
     parseval = float(ny / (N * nx) - 1)
 
+    cufft_comp = cufft_comparator(x, flush, min(args.steps, 50)) if world == 1 else None
     if rank != 0:
         return
     peaks = load_peaks()
@@ -355,13 +382,19 @@ def run_fmmfft(args, rank, world, local_rank):
         alu_peak = 148 * 64 * 2 * sm_max * 1e6 / 1e12         # FP64 FMA lanes (half rate)
     hbm_peak = peaks.get("hbm_gbs", 6454.3)
     rl = {}
+    # 3xTF32 on tcgen05: the measured dense bf16 peak x 1/2 (tf32 : bf16 nominal) / 3 passes
+    tc_peak = peaks.get("bf16_tflops", 1673.2) * 0.5 / 3
+    v = info["variant"]
+    mk = "k_fft_rowc" if v & 16 else "k_fft_row" if v & 4 else "k_fft_col + k_fft_rowt" if v & 8 else "k_fft_pass"
     for st_name, (kname, bound, amount) in stage_rooflines(N, P, B, Q, M_L, G, info["L"], prec,
-                                                           bool(info["variant"] & 1)).items():
+                                                           bool(info["variant"] & 1), bool(info["variant"] & 2), mk).items():
         t = stages.get(st_name)
         if not t or t != t:
             continue
         if bound == "alu":
             ach, pk, unit = amount / (t * 1e-3) / 1e12, alu_peak, "TFLOP/s"
+        elif bound == "tensor":
+            ach, pk, unit = amount / (t * 1e-3) / 1e12, tc_peak, "TFLOP/s"
         else:
             ach, pk, unit = amount / (t * 1e-3) / 1e9, hbm_peak, "GB/s"
         rl[st_name] = {"kernel": kname, "bound": bound, "achieved": ach, "peak": pk, "unit": unit, "frac": ach / pk,
@@ -370,7 +403,9 @@ def run_fmmfft(args, rank, world, local_rank):
     dom = max(rl, key=lambda k: rl[k]["avg_launch_ms"])
     roof = dict(rl[dom], stage=dom,
                 peak_basis=(f"148 SMs x {'128 FP32' if prec == 'c64' else '64 FP64'} FMA/clk x 2 x {sm_max} MHz (guide unit counts)"
-                            if rl[dom]["bound"] == "alu" else "MEASURED_PEAKS.json HBM copy bandwidth"))
+                            if rl[dom]["bound"] == "alu" else
+                            "MEASURED_PEAKS.json bf16 dense x 0.5 (tf32 nominal ratio) / 3 (3xTF32)" if rl[dom]["bound"] == "tensor"
+                            else "MEASURED_PEAKS.json HBM copy bandwidth"))
     clocks = sampler.summary()
     line = {
         "metric": "1D C2C FFT GFLOP/s (5N log2N/t)", "value": value, "unit": "GFLOP/s", "n_gpus": world,
@@ -388,6 +423,8 @@ def run_fmmfft(args, rank, world, local_rank):
         "gpu_launches": info["kernels_per_execute"] * args.steps,
         "clocks": {k: clocks[k] for k in ("sm_mhz", "sm_max_mhz", "reasons")},
     }
+    if world == 1:
+        line["comparator"] = cufft_comp
     if world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(workload, G)
     print(json.dumps(line), flush=True)

@@ -68,6 +68,11 @@ typedef enum {
                                    returns. Without it the fused single-GPU far field
                                    (FMMFFT_VARIANT_TREE_FUSED) keeps levels < L on chip only, and
                                    those debug buffers hold stale data. */
+#define FMMFFT_FLAG_INVERSE 8u  /* the inverse transform x_j = (1/N) sum_k y_k exp(+2 pi i jk/N)
+                                   (F_N^{-1} = F_N^H / N): the same FMM-FFT
+                                   path on conj(input), its output conjugated and scaled by 1/N
+                                   (two extra elementwise passes, k_conj_scale). Same layouts,
+                                   distribution and error bounds as the forward plan. */
 
 /* ---------------------------------------------------------------- communicator (G > 1)
  * One process per GPU. Rank 0 calls fmmfft_get_unique_id and broadcasts the 128 bytes (e.g.
@@ -125,6 +130,9 @@ typedef struct {
 #define FMMFFT_VARIANT_TREE_FUSED 1u  /* far field as one per-FMM kernel (G = 1, tree fits smem) */
 #define FMMFFT_VARIANT_S2T_TC     2u  /* near field on tcgen05 tensor cores (3xTF32)             */
 #define FMMFFT_VARIANT_ROW_FFT1   4u  /* M-point FFTs as one single-pass kernel per row        */
+#define FMMFFT_VARIANT_FOURSTEP   8u  /* long rows: column pass(es) + transposing row pass     */
+#define FMMFFT_VARIANT_ROW_CL    16u  /* rows split over a cluster of CTAs (k_fft_rowc)        */
+#define FMMFFT_VARIANT_DOWN_LVL  32u  /* wide levels on the per-level M2M / M2L kernels        */
 
 FMMFFT_API fmmfft_status_t fmmfft_get_info(fmmfft_plan_t plan, fmmfft_info_t* info);
 

@@ -173,6 +173,7 @@ struct RankBufs {
     void* haloL = nullptr;   // S box -1  (G > 1)
     void* haloR = nullptr;   // S box nb  (G > 1)
     void* r = nullptr;       // [P] reductions
+    void* cin = nullptr;     // conj(in) (inverse plans)
     void* din = nullptr;     // execute_host staging
     void* dout = nullptr;
     std::vector<void*> Mpad, Lloc, Mfull, Lfull;   // indexed by level
@@ -210,6 +211,8 @@ struct fmmfft_plan_s {
     int tree_cl = 1;                 // k_tree_pc: CTAs per FMM (cluster), 1 = not used
     bool tree_phased = false;        // ... as up / all-levels M2L / L2L-chain launches (FMMFFT_TREE=p) (k_tree_pq<.., false>, k_m2l_flat, k_tree_dn)
     int fs_lc1 = 0, fs_lc2 = 0, fs_lr = 0;   // four-step large-M FFT: column pass bits (2nd: 0 = none), row pass bits
+    int s2m_nbx = 0, s2m_pc = 0, pp_ms = 0;  // tuning knobs (FMMFFT_S2M_NBX, FMMFFT_S2M_PC, FMMFFT_PP_MS); 0 = default
+    bool inverse = false;            // FMMFFT_FLAG_INVERSE: x = F_N^{-1} y
     bool lvl_off = false;            // FMMFFT_DOWN=tree: every down level in k_tree_down (no k_m2l_lvl)
     bool s2t_tc = false;             // S2T on tcgen05 (k_s2t_tc): complex64, M_L = 64, nb % 128 == 0
     void* toep = nullptr;            // its Toeplitz hi/lo operand table
@@ -404,6 +407,7 @@ static fmmfft_status_t alloc_rank(fmmfft_plan_s* p, RankBufs& rb) {
     if ((st = dalloc(p, &rb.W, n_local * e))) return st;
     if ((st = dalloc(p, &rb.tmp, n_local * e))) return st;
     if (p->s2t_tc && (st = dalloc(p, &rb.Sp, n_local * e))) return st;
+    if (p->inverse && (st = dalloc(p, &rb.cin, n_local * e))) return st;
     if (p->G > 1) {
         if ((st = dalloc(p, &rb.Rcv, n_local * e))) return st;
         if ((st = dalloc(p, &rb.haloL, (size_t)p->M_L * p->P * e))) return st;
@@ -628,11 +632,13 @@ struct Exec {
     // post_pfft), so the far field and the near field run concurrently
     fmmfft_status_t near_up() {
         fmmfft_status_t st;
-        const int PCs = std::min(p->P, sizeof(R) == 4 ? 32 : 16);
+        const int PCs = std::min(p->P, p->s2m_pc ? p->s2m_pc : (sizeof(R) == 4 ? 32 : 16));
         for (RankBufs& rb : p->ranks) {
             const C* S = in[p->virt ? rb.g : 0];
             const int Qp = (p->Q + 3) / 4 * 4;
-            const int nbx = p->nb >= 2 ? 2 : 1;                // boxes per CTA (k_s2m NBX = 2; nb is even or 1)
+            // boxes per CTA (k_s2m NBX <= 2; nb is even or 1): 1 unless that gives > 4 CTAs per SM
+            int nbx = p->s2m_nbx ? p->s2m_nbx : ((long long)p->nb * (p->P / PCs) > 4 * 148 ? 2 : 1);
+            if (p->nb < 2) nbx = 1;
             const size_t smem = (size_t)2 * p->M_L * (PCs + 1) * sizeof(C) + (size_t)Qp * p->M_L * sizeof(R);
             const dim3 grid((unsigned)(p->nb / nbx), (unsigned)(p->P / PCs));
             dispatch<2, 4, 8, 16, 32>(PCs, [&](auto pc) {
@@ -1050,7 +1056,11 @@ struct Exec {
 
     // ---- L2T + POST + P-FFT
     fmmfft_status_t post_pfft() {
-        const int MS = std::min(p->M_L, std::max(1, TILE / p->P));
+        // m sub-tile per CTA: the whole P-point FFT tile, split further (down to 16) while that
+        // leaves fewer than ~4 CTAs per SM (small N: latency-bound, more CTAs in flight)
+        int MS = std::min(p->M_L, std::max(1, TILE / p->P));
+        while (MS > 16 && (long long)p->nb * (p->M_L / MS) < 4 * 148) MS /= 2;
+        if (p->pp_ms) MS = std::min(p->M_L, p->pp_ms);
         const int threads = std::min(sizeof(R) == 4 ? 1024 : 512, std::max(32, MS * p->P / 8));
         size_t smem = (size_t)MS * (p->P + 1) * sizeof(C) + (size_t)p->P * sizeof(C) + (size_t)p->Q * MS * sizeof(R);
         const int stage_L = smem + (size_t)p->Q * p->P * sizeof(C) <= 160 * 1024;   // stage L^L of the box
@@ -1201,7 +1211,33 @@ struct Exec {
         return FMMFFT_SUCCESS;
     }
 
+    // inverse plans: y <- scale * conj(x) over this rank's N/G elements
+    fmmfft_status_t conj_scale(const C* x, C* y, R scale) {
+        const long long n = p->N / p->G;
+        const unsigned blocks = (unsigned)std::min<long long>((n / 2 + 255) / 256, 148LL * 8);
+        launch_pdl(k_conj_scale<R>, blocks, 256, 0, s, x, y, n, scale);
+        LAUNCH_CHECK();
+        return FMMFFT_SUCCESS;
+    }
+
     fmmfft_status_t run() {
+        fmmfft_status_t st;
+        if (p->inverse)                                 // F^{-1} x = conj(F conj(x)) / N
+            for (RankBufs& rb : p->ranks) {
+                const int g = p->virt ? rb.g : 0;
+                if ((st = conj_scale(in[g], (C*)rb.cin, R(1)))) return st;
+                in[g] = (const C*)rb.cin;
+            }
+        if ((st = run_forward())) return st;
+        if (p->inverse)
+            for (RankBufs& rb : p->ranks) {
+                const int g = p->virt ? rb.g : 0;
+                if ((st = conj_scale(out[g], out[g], R(1) / (R)p->N))) return st;
+            }
+        return FMMFFT_SUCCESS;
+    }
+
+    fmmfft_status_t run_forward() {
         fmmfft_status_t st;
 #define STEP(stage, call) if ((st = mark(stage))) return st; if ((st = call)) return st;
         STEP(ST_COMM_S, comm_S())
@@ -1357,6 +1393,7 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
 
     fmmfft_plan_s* p = new fmmfft_plan_s;
     p->N = N; p->P = P; p->G = G; p->B = B; p->Q = Q; p->M_L = M_L; p->L = L;
+    p->inverse = (flags & FMMFFT_FLAG_INVERSE) != 0;
     p->M = N / P; p->Mg = p->M / G; p->prec = precision; p->flags = flags; p->virt = virt; p->device = dev;
     p->nb = (int)(nleaf / G);
     p->lg = std::min(std::max(B, ilog2(G) + 1), L);
@@ -1390,6 +1427,9 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
     p->s2t_tc = precision == FMMFFT_C64 && M_L == 64 && (p->nb % S2TC_BOXES) == 0;
     if (const char* e = getenv("FMMFFT_S2T")) p->s2t_tc = p->s2t_tc && e[0] == 't';
     if (const char* e = getenv("FMMFFT_DOWN")) p->lvl_off = e[0] == 't';
+    if (const char* e = getenv("FMMFFT_S2M_NBX")) p->s2m_nbx = atoi(e) == 1 ? 1 : 2;
+    if (const char* e = getenv("FMMFFT_S2M_PC")) { const int v = atoi(e); if (v == 8 || v == 16 || (v == 32 && precision == FMMFFT_C64)) p->s2m_pc = v; }
+    if (const char* e = getenv("FMMFFT_PP_MS")) { const int v = atoi(e); if (v >= 8 && v <= M_L && pow2(v)) p->pp_ms = v; }
     const char* g_env = getenv("FMMFFT_NO_GRAPH");
     p->use_graph = !(g_env && g_env[0] == '1');
     plan_radices(p);
@@ -1411,6 +1451,10 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
         const int mx = precision == FMMFFT_C64 ? 11 : 10;
         const char* e = getenv("FMMFFT_MFFT");
         const bool want = !(e && e[0] == 'p') && !(getenv("FMMFFT_ROWFFT") && getenv("FMMFFT_ROWFFT")[0] == '0');
+        // FMMFFT_MFFT=fs forces it; by default also rows of >= 2^13 points when there are fewer rows
+        // than SMs (k_fft_row would run one CTA per row on part of the GPU)
+        const bool few_rows = P / G < 148 && lM >= 13 && !getenv("FMMFFT_ROWFFT_CL") && !(e && e[0] == 'r');
+        if (want && ((e && e[0] == 'f' && lM >= 10) || few_rows)) { p->row_fft1 = false; p->row_cl = 0; }
         if (want && !p->row_fft1 && !p->row_cl && lM >= 10 && lM <= 3 * mx) {
             if (lM <= 2 * mx) {
                 p->fs_lr = std::min(mx, (lM + 1) / 2);
@@ -1515,7 +1559,8 @@ fmmfft_status_t fmmfft_get_info(fmmfft_plan_t p, fmmfft_info_t* info) {
     info->L = p->L; info->precision = p->prec; info->M = p->M; info->level_gather = p->lg;
     info->n_stages = ST_COUNT + 1; info->workspace_bytes = p->ws_bytes; info->kernels_per_execute = p->kernels;
     info->variant = (p->tree_p ? FMMFFT_VARIANT_TREE_FUSED : 0u) | (p->s2t_tc ? FMMFFT_VARIANT_S2T_TC : 0u) |
-                    ((p->row_fft1 || p->row_cl) ? FMMFFT_VARIANT_ROW_FFT1 : 0u);
+                    ((p->row_fft1 || p->row_cl) ? FMMFFT_VARIANT_ROW_FFT1 : 0u) | (p->fs_lr ? FMMFFT_VARIANT_FOURSTEP : 0u) |
+                    (p->row_cl ? FMMFFT_VARIANT_ROW_CL : 0u) | (!p->tree_p && !p->lvl_off ? FMMFFT_VARIANT_DOWN_LVL : 0u);
     return FMMFFT_SUCCESS;
 }
 

@@ -706,4 +706,29 @@ k_fft_rowt(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, long long M, i
     for (int t = 0; t < 16; ++t) y[(long long)(j + t * NT) << lrpr] = v[t];
 }
 
+
+// ---------------------------------------------------------------------------------------------
+// Inverse transform (§8(f) NEXT-1): F_N^{-1} x = conj(F_N conj(x)) / N (F_N^{-1} = F_N^H / N),
+// so the inverse plan conjugates its input into a workspace copy, runs the forward path and
+// conjugates and scales the output in place: out[i] = scale * conj(in[i]). Two complex values
+// per thread-iteration as one 16- (c64) or two 16-byte (c128) accesses.
+// ---------------------------------------------------------------------------------------------
+template <typename R>
+__global__ void __launch_bounds__(256)
+k_conj_scale(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, long long n, R scale) {
+    pdl_trigger();
+    pdl_wait();
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; 2 * i < n; i += stride) {
+        if constexpr (sizeof(R) == 4) {
+            const float4 v = __ldg(reinterpret_cast<const float4*>(in) + i);
+            reinterpret_cast<float4*>(out)[i] = make_float4(scale * v.x, -scale * v.y, scale * v.z, -scale * v.w);
+        } else {
+            const double2 a = __ldg(in + 2 * i), b = __ldg(in + 2 * i + 1);
+            out[2 * i] = make_double2(scale * a.x, -scale * a.y);
+            out[2 * i + 1] = make_double2(scale * b.x, -scale * b.y);
+        }
+    }
+}
+
 }  // namespace fmmfft

@@ -15,7 +15,7 @@ import ctypes
 import torch
 
 from . import _lib
-from ._lib import C64, C128, FLAG_DEBUG, FLAG_PROFILE, FLAG_VIRTUAL, check, lib
+from ._lib import C64, C128, FLAG_DEBUG, FLAG_INVERSE, FLAG_PROFILE, FLAG_VIRTUAL, check, lib
 
 _DT = {"c64": (C64, torch.complex64), "c128": (C128, torch.complex128)}
 
@@ -58,12 +58,15 @@ class _DevView:
 
 class FmmFFT:
     def __init__(self, N: int, P: int, G: int = 1, B: int = 2, Q: int = 16, precision: str = "c64",
-                 M_L: int = 64, virtual: bool = False, profile: bool = False, debug: bool = False):
+                 M_L: int = 64, virtual: bool = False, profile: bool = False, debug: bool = False,
+                 inverse: bool = False):
         self.N, self.P, self.G, self.B, self.Q, self.M_L = N, P, G, B, Q, M_L
         self.precision = precision
         self.virtual = virtual
         self._prec, self.dtype = _DT[precision]
-        flags = (FLAG_VIRTUAL if virtual else 0) | (FLAG_PROFILE if profile else 0) | (FLAG_DEBUG if debug else 0)
+        flags = (FLAG_VIRTUAL if virtual else 0) | (FLAG_PROFILE if profile else 0) | (FLAG_DEBUG if debug else 0) | \
+                (FLAG_INVERSE if inverse else 0)
+        self.inverse = inverse
         h = ctypes.c_void_p()
         check(lib.fmmfft_plan_ex(ctypes.byref(h), N, P, G, B, Q, self._prec, M_L, flags))
         self._h = h

@@ -268,3 +268,22 @@ def test_large_m_fft(F, monkeypatch, N, P, prec, G, env):
         monkeypatch.setenv(k, v)
     plan, x, y = run(F, N, P, 2, 16, prec, 64, G=G, virtual=G > 1)
     assert rel(y, O.fft_radix2(x)) < TOL_E2E[prec]
+
+
+# ------------------------------------------------------------------ inverse transform (§8(f) NEXT-1)
+@pytest.mark.parametrize("N,P,B,Q,prec,M_L,G", [
+    (1 << 12, 16, 2, 16, "c128", 64, 1),
+    (1 << 20, 64, 2, 16, "c64", 64, 1),       # the cfg2 shape
+    (1 << 20, 16, 3, 16, "c128", 16, 2),      # distributed (virtual ranks)
+    (1 << 23, 2, 2, 16, "c64", 64, 1),        # four-step M-FFT
+])
+def test_inverse_vs_oracle(F, N, P, B, Q, prec, M_L, G):
+    x = SI.complex_uniform(0, N, dtype=NPDT[prec])
+    inv = F(N=N, P=P, G=G, B=B, Q=Q, precision=prec, M_L=M_L, virtual=G > 1, inverse=True)
+    y = inv(torch.from_numpy(x).cuda()).cpu().numpy()
+    ref = O.dft_direct(x, inverse=True) if N <= 1 << 12 else O.fft_radix2(x, inverse=True)
+    assert rel(y, ref) < TOL_E2E[prec]
+    # round trip forward -> inverse
+    fwd = F(N=N, P=P, G=G, B=B, Q=Q, precision=prec, M_L=M_L, virtual=G > 1)
+    z = inv(fwd(torch.from_numpy(x).cuda())).cpu().numpy()
+    assert rel(z, x) < 2 * TOL_E2E[prec]

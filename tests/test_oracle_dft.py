@@ -120,3 +120,26 @@ def test_fft2d_layout_against_library():
     Y = np.fft.fft2(T.reshape(M, P))            # Y[k1, k2]
     expect = Y.T.reshape(M * P)                 # index k1 + M k2
     assert O.rel_l2(O.fft2d_MP(T, M, P), expect) < 1e-14
+
+
+# ------------------------------------------------------------------ the inverse transform (§8(f) NEXT-1)
+def test_inverse_closed_forms():
+    N = 64
+    # F^{-1} delta_0 = 1/N (constant); F^{-1} delta_k0 = tone w_N^{-j k0} / N
+    d = np.zeros(N, complex)
+    d[0] = 1
+    assert np.allclose(O.dft_direct(d, inverse=True), np.full(N, 1 / N), atol=1e-16)
+    d[:] = 0
+    d[5] = 1
+    j = np.arange(N)
+    assert np.allclose(O.dft_direct(d, inverse=True), np.exp(2j * np.pi * 5 * j / N) / N, atol=1e-16)
+
+
+@pytest.mark.parametrize("N", [2, 16, 256, 4096])
+def test_inverse_roundtrip_and_radix2(N):
+    x = SI.complex_uniform(0, N)
+    y = O.dft_direct(x)
+    assert O.rel_l2(O.dft_direct(y, inverse=True), x) < 1e-13
+    assert O.rel_l2(O.fft_radix2(y, inverse=True), x) < 1e-13
+    assert O.rel_l2(O.fft_radix2(x, inverse=True), O.dft_direct(x, inverse=True)) < 1e-13
+    assert O.rel_l2(O.fft_radix2(x, inverse=True), np.fft.ifft(x)) < 1e-13
