@@ -68,6 +68,11 @@ typedef enum {
                                    returns. Without it the fused single-GPU far field
                                    (FMMFFT_VARIANT_TREE_FUSED) keeps levels < L on chip only, and
                                    those debug buffers hold stale data. */
+#define FMMFFT_FLAG_DIRECT 16u  /* no FMM: the plain four-step (Cooley-Tukey) FFT of length N with
+                                   the same M-FFT kernels, as the in-house comparator (SURVEY §8(f)
+                                   NEXT-3). G = 1 only (else FMMFFT_UNSUPPORTED); P, B, Q, M_L are
+                                   ignored; 2^10 <= N <= 2^33 (c64) / 2^30 (c128); combinable with
+                                   FMMFFT_FLAG_INVERSE. */
 #define FMMFFT_FLAG_INVERSE 8u  /* the inverse transform x_j = (1/N) sum_k y_k exp(+2 pi i jk/N)
                                    (F_N^{-1} = F_N^H / N): the same FMM-FFT
                                    path on conj(input), its output conjugated and scaled by 1/N
@@ -90,7 +95,7 @@ FMMFFT_API fmmfft_status_t fmmfft_comm_destroy(void);
  * Requirements (else FMMFFT_INVALID_VALUE):
  *   N, P, M_L powers of two; P >= 2; G in {1, 2, 4, 8}; P % G == 0; N % (P M_L) == 0;
  *   L = log2(N / (P M_L)) >= B >= 2; 2^L % G == 0; 2 <= Q <= 32;
- *   16 <= M_L <= 256; P <= 2048; M = N / P >= 2 G.
+ *   16 <= M_L <= 128; P <= 1024 (complex64) / 512 (complex128); M = N / P >= 2 G.
  *   Without FMMFFT_FLAG_VIRTUAL and G > 1, fmmfft_comm_init must have been called with the
  *   same G (else FMMFFT_NOT_INITIALIZED). The device must be sm_100 (else UNSUPPORTED).
  * Collective when G > 1 (non-virtual): every rank creates its plan with identical arguments.
@@ -100,6 +105,31 @@ FMMFFT_API fmmfft_status_t fmmfft_plan(fmmfft_plan_t* plan, long long N, int P, 
                             fmmfft_precision_t precision);
 FMMFFT_API fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, int B, int Q,
                                fmmfft_precision_t precision, int M_L, unsigned flags);
+
+/* ---------------------------------------------------------------- parameter autotuner
+ * pick (P, B, Q, M_L) for (N, G, precision) and a relative-l2 error target
+ * `tol` (the paper searches its parameter space per N, Figs. 6-9).
+ *   Q: the smallest of {8, 16, 24} whose predicted error meets tol with a 4x margin — the
+ *      truncation model e(Q) = 1.7e-3 * 6.3^-(Q-2) fitted to the oracle's Q sweep (DESIGN.md §2,
+ *      geometric decay, saturating near Q = 18) — plus the arithmetic floor
+ *      (2.6e-7 complex64, 3e-14 complex128). FMMFFT_INVALID_VALUE if no Q reaches tol.
+ *   M_L = 64 (the tensor-core S2T's tile), P over the powers of two with G | P,
+ *      L = log2(N/(P M_L)) >= B and G | 2^L, B over {2, 3, 4} (B <= L).
+ *   measure != 0 (G = 1 only): every candidate plan is built and timed on the current device
+ *      (3 warm-up + 5 timed executes, CUDA events, on a scratch input) — the fastest wins;
+ *      measure == 0: ranked by a roofline model (HBM passes, tensor / FFMA2 flops, per-launch
+ *      latency), host only, no device work.
+ * best->ms is the measured (or modelled) time of the winner, best->error its predicted error,
+ * best->candidates the number of (P, B) pairs considered. */
+typedef struct {
+    int P, B, Q, M_L;
+    float ms;
+    double error;
+    int candidates;
+} fmmfft_tune_t;
+
+FMMFFT_API fmmfft_status_t fmmfft_autotune(long long N, int G, fmmfft_precision_t precision, double tol, int measure,
+                                           fmmfft_tune_t* best);
 
 /* Forward transform. in, out: device pointers on the plan's device, N/G complex elements
  * each (N for a virtual plan), 16-byte aligned, non-overlapping (else INVALID_VALUE).

@@ -13,13 +13,13 @@ SUCCESS, INVALID_VALUE, UNSUPPORTED, ALLOC_FAILED, CUDA_ERROR, NCCL_ERROR, NOT_I
 STATUS_NAMES = ["SUCCESS", "INVALID_VALUE", "UNSUPPORTED", "ALLOC_FAILED", "CUDA_ERROR", "NCCL_ERROR",
                 "NOT_INITIALIZED"]
 C64, C128 = 0, 1
-FLAG_VIRTUAL, FLAG_PROFILE, FLAG_DEBUG, FLAG_INVERSE = 1, 2, 4, 8
+FLAG_VIRTUAL, FLAG_PROFILE, FLAG_DEBUG, FLAG_INVERSE, FLAG_DIRECT = 1, 2, 4, 8, 16
 
 # every symbol include/fmmfft.h declares (checked by tests/test_abi.py)
 EXPORTS = [
     "fmmfft_get_unique_id", "fmmfft_comm_init", "fmmfft_comm_destroy", "fmmfft_plan", "fmmfft_plan_ex",
     "fmmfft_execute", "fmmfft_execute_host", "fmmfft_destroy", "fmmfft_get_info", "fmmfft_stage_times",
-    "fmmfft_stage_name", "fmmfft_debug_buffer", "fmmfft_last_error", "fmmfft_version",
+    "fmmfft_stage_name", "fmmfft_debug_buffer", "fmmfft_last_error", "fmmfft_version", "fmmfft_autotune",
 ]
 
 
@@ -29,6 +29,11 @@ class Info(ctypes.Structure):
                 ("M", ctypes.c_longlong), ("level_gather", ctypes.c_int), ("n_stages", ctypes.c_int),
                 ("workspace_bytes", ctypes.c_size_t), ("kernels_per_execute", ctypes.c_int),
                 ("variant", ctypes.c_uint)]
+
+
+class Tune(ctypes.Structure):
+    _fields_ = [("P", ctypes.c_int), ("B", ctypes.c_int), ("Q", ctypes.c_int), ("M_L", ctypes.c_int),
+                ("ms", ctypes.c_float), ("error", ctypes.c_double), ("candidates", ctypes.c_int)]
 
 
 class FmmfftError(RuntimeError):
@@ -59,6 +64,7 @@ def _load() -> ctypes.CDLL:
         "fmmfft_debug_buffer": (st, [vp, i, i, i, ctypes.POINTER(vp), ctypes.POINTER(ctypes.c_size_t)]),
         "fmmfft_last_error": (ctypes.c_char_p, []),
         "fmmfft_version": (ctypes.c_char_p, []),
+        "fmmfft_autotune": (st, [ll, i, i, ctypes.c_double, i, ctypes.POINTER(Tune)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)

@@ -213,6 +213,8 @@ struct fmmfft_plan_s {
     int fs_lc1 = 0, fs_lc2 = 0, fs_lr = 0;   // four-step large-M FFT: column pass bits (2nd: 0 = none), row pass bits
     int s2m_nbx = 0, s2m_pc = 0, pp_ms = 0;  // tuning knobs (FMMFFT_S2M_NBX, FMMFFT_S2M_PC, FMMFFT_PP_MS); 0 = default
     bool inverse = false;            // FMMFFT_FLAG_INVERSE: x = F_N^{-1} y
+    bool pp_old = false;             // FMMFFT_PP=tile: the shared-memory-tile k_post_pfft for every P
+    bool direct = false;             // FMMFFT_FLAG_DIRECT: plain four-step FFT of length N, no FMM
     bool lvl_off = false;            // FMMFFT_DOWN=tree: every down level in k_tree_down (no k_m2l_lvl)
     bool s2t_tc = false;             // S2T on tcgen05 (k_s2t_tc): complex64, M_L = 64, nb % 128 == 0
     void* toep = nullptr;            // its Toeplitz hi/lo operand table
@@ -383,7 +385,7 @@ static constexpr int kTileF = 8192, kTileD = 4096;   // shared FFT tile (element
 template <typename R> static constexpr int kRowFftMax = sizeof(R) == 4 ? 14 : 13;   // k_fft_row: whole row in smem
 // four-step passes: largest pass length (log2) and columns (rows) per CTA for a pass of 2^l points
 template <typename R> __host__ __device__ constexpr int fs_max() { return sizeof(R) == 4 ? 11 : 10; }
-template <typename R> __host__ __device__ constexpr int fs_cols(int l) { return l <= fs_max<R>() - 1 ? 16 : 8; }
+template <typename R> __host__ __device__ constexpr int fs_cols(int l) { return l <= fs_max<R>() - 2 ? 16 : 8; }
 
 static void plan_radices(fmmfft_plan_s* p) {
     const int maxbits = p->prec == FMMFFT_C64 ? 10 : 9;
@@ -396,6 +398,22 @@ static void plan_radices(fmmfft_plan_s* p) {
         p->radices.push_back(1 << b);
         left -= b;
     }
+}
+
+// four-step split of a 2^lM-point row into passes of <= 2^mx points (2 or 3 passes; none if the
+// row is too short or too long)
+static void choose_fourstep(fmmfft_plan_s* p, int lM, int mx) {
+    p->fs_lr = p->fs_lc1 = p->fs_lc2 = 0;
+    if (lM < 10 || lM > 3 * mx) return;
+    if (lM <= 2 * mx) {
+        p->fs_lr = std::min(mx, (lM + 1) / 2);
+        p->fs_lc1 = lM - p->fs_lr;
+    } else {
+        p->fs_lr = std::min(mx, (lM + 2) / 3);
+        p->fs_lc1 = std::min(mx, (lM - p->fs_lr + 1) / 2);
+        p->fs_lc2 = lM - p->fs_lr - p->fs_lc1;
+    }
+    if (p->fs_lc1 < 5 || p->fs_lr < 5 || (p->fs_lc2 && p->fs_lc2 < 5)) p->fs_lr = p->fs_lc1 = p->fs_lc2 = 0;
 }
 
 static fmmfft_status_t alloc_rank(fmmfft_plan_s* p, RankBufs& rb) {
@@ -500,6 +518,13 @@ static fmmfft_status_t init_kernel_attrs() {
             set((const void*)k_tree_pc<8, 256, 4>);
         }
         if constexpr (sizeof(R) == 4) set((const void*)k_s2t_tc);
+        set((const void*)k_base_sg<R, 4, sizeof(R) == 4 ? 8 : 4, 4>);
+        for (int lp = 1; lp <= 5; ++lp)
+            dispatch<1, 2, 3, 4, 5>(lp, [&](auto v) {
+                set((const void*)k_post_pfft_r<R, decltype(v)::value, 8>);
+                set((const void*)k_post_pfft_r<R, decltype(v)::value, 16>);
+                set((const void*)k_post_pfft_r<R, decltype(v)::value, 24>);
+            });
         set((const void*)k_m2l_lvl<R, 8>);
         set((const void*)k_m2m_lvl<R, 8>);
         set((const void*)k_m2m_lvl<R, 16>);
@@ -661,8 +686,10 @@ struct Exec {
                 CUDA_TRY(cudaStreamWaitEvent(p->side, p->fork2, 0));
                 if ((st = mark_on(p->ev_s2t[0], p->side))) return st;
                 const int ntile = p->nb / S2TC_BOXES;
-                int tpc = 1;                                       // tiles per CTA: about one wave
-                while (tpc < ntile && (long long)(ntile / tpc) * (p->P - 1) > 148) tpc *= 2;
+                // tiles per CTA: the fewest that keep the grid within one wave of 148 SMs
+                // (one CTA per SM: TMEM + ~180 KB of shared memory)
+                const int cpp = std::max(1, 148 / (p->P - 1));             // CTAs per p
+                const int tpc = (ntile + cpp - 1) / cpp;
                 for (RankBufs& rb : p->ranks) {
                     const dim3 grid((unsigned)((ntile + tpc - 1) / tpc), (unsigned)(p->P - 1));
                     launch_pdl(k_s2t_tc, grid, S2TC_THREADS, s2tc_smem_bytes(), p->side, (const C*)rb.Sp, (const C*)rb.haloL,
@@ -722,7 +749,8 @@ struct Exec {
         const bool lvl_ok = !p->lvl_off && (p->Q == 8 || p->Q == 16 || p->Q == 24) && p->PCd % PCl == 0 && p->P % PCl == 0;
         int optin = 0;
         CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, p->device));
-        while (lvl_ok && cur > to && (nbc >> 1) >= 2 * lvl_nt<R, 16>()) {
+        while (lvl_ok && cur > to && (nbc >> 1) >= 2 * lvl_nt<R, 16>() &&
+               (long long)((nbc >> 1) / lvl_nt<R, 16>()) * (p->P / PCl) >= 148) {
             C* o = (C*)outs(cur - 1);
             const int nsub = p->P / PCl;
             dispatch<8, 16, 24>(p->Q, [&](auto qv) {
@@ -900,6 +928,18 @@ struct Exec {
     // M2L-B + REDUCE on the gathered base level (sources: all 2^B boxes, periodic)
     fmmfft_status_t launch_base(RankBufs& rb, C* outp, long long tgt_base, int ntg) {
         const int nbB = 1 << p->B;
+        {   // all shifts staged at once, shift groups in parallel (k_base_sg)
+            constexpr int PCb = sizeof(R) == 4 ? 8 : 4, SG = 4, NTb = 4;
+            const size_t smem = (size_t)nbB * p->Q * PCb * sizeof(C) + (size_t)SG * NTb * p->Q * PCb * sizeof(C) +
+                                (size_t)(nbB - 3) * p->Q * p->Q * PCb * sizeof(R);
+            if (nbB >= 4 && p->PCd % PCb == 0 && p->P % PCb == 0 && smem <= 200 * 1024 && PCb * p->Q * SG <= 1024) {
+                const dim3 grid((unsigned)(p->P / PCb), (unsigned)((ntg + NTb - 1) / NTb));
+                launch_pdl(k_base_sg<R, NTb, PCb, SG>, grid, PCb * p->Q * SG, smem, s, (const C*)rb.Mfull[p->B], outp,
+                           (C*)rb.r, (int)tgt_base, ntg, (const R*)p->m2lB, p->m2lB_chunk, p->PCd, nbB, p->P, p->Q);
+                LAUNCH_CHECK();
+                return FMMFFT_SUCCESS;
+            }
+        }
         const int PC_ = p->PCd;
         const size_t smem = ((size_t)nbB + 1) * p->Q * PC_ * sizeof(C) + (size_t)p->Q * p->Q * PC_ * sizeof(R);
         if (ntg <= 32 && smem <= 200 * 1024) {
@@ -973,8 +1013,11 @@ struct Exec {
         if (!(p->Q == 8 || p->Q == 16 || p->Q == 24)) return p->L + 1;
         constexpr int PCl = lvl_pc<R>();
         if (p->PCd % PCl || p->P % PCl) return p->L + 1;
+        // a level goes to k_m2l_lvl once its tiles x p sub-chunks fill the GPU; narrower levels
+        // are latency-bound there (one tile per CTA) and cheaper inside k_tree_down's single launch
+        const int nsub = p->P / PCl;
         for (int lev = std::max(p->B, p->lg) + 1; lev <= p->L; ++lev)
-            if (nb_at(lev) >= 2 * lvl_nt<R, 16>()) return lev;
+            if (nb_at(lev) >= 2 * lvl_nt<R, 16>() && (long long)(nb_at(lev) / lvl_nt<R, 16>()) * nsub >= 148) return lev;
         return p->L + 1;
     }
 
@@ -1056,6 +1099,26 @@ struct Exec {
 
     // ---- L2T + POST + P-FFT
     fmmfft_status_t post_pfft() {
+        // P <= 32 (and a specialised Q): the register-resident variant, one thread per (box, m)
+        if (p->P <= 32 && p->P >= 2 && (p->Q == 8 || p->Q == 16 || p->Q == 24) && p->M_L <= 256 && !p->pp_old) {
+            const int nbx = std::max(1, std::min(p->nb, 256 / p->M_L));
+            if (p->nb % nbx == 0) {
+                const size_t smem = ((size_t)nbx * p->Q * p->P + 2 * p->P + 16) * sizeof(C);
+                for (RankBufs& rb : p->ranks) {
+                    bool ok = dispatch<1, 2, 3, 4, 5>(ilog2(p->P), [&](auto lp) {
+                        constexpr int LP = decltype(lp)::value;
+                        dispatch<8, 16, 24>(p->Q, [&](auto qv) {
+                            launch_pdl(k_post_pfft_r<R, LP, decltype(qv)::value>, (unsigned)(p->nb / nbx), nbx * p->M_L, smem, s,
+                                       (const C*)rb.Tn, (const C*)rb.Lloc[p->L], (const C*)rb.r, (const C*)p->rho,
+                                       (const R*)p->s2m, (C*)rb.W, ilog2(p->M_L), (int)p->Mg);
+                        });
+                    });
+                    if (!ok) return fail(FMMFFT_UNSUPPORTED, "k_post_pfft_r: P=%d", p->P);
+                    LAUNCH_CHECK();
+                }
+                return FMMFFT_SUCCESS;
+            }
+        }
         // m sub-tile per CTA: the whole P-point FFT tile, split further (down to 16) while that
         // leaves fewer than ~4 CTAs per SM (small N: latency-bound, more CTAs in flight)
         int MS = std::min(p->M_L, std::max(1, TILE / p->P));
@@ -1128,7 +1191,7 @@ struct Exec {
         const int lM = ilog2(p->M);
         for (RankBufs& rb : p->ranks) {
             C* dst = out[p->virt ? rb.g : 0];
-            const C* src = (const C*)(p->G > 1 ? rb.Rcv : rb.W);
+            const C* src = p->direct ? in[0] : (const C*)(p->G > 1 ? rb.Rcv : rb.W);
             if (p->fs_lr) {                      // four-step: column pass(es) + transposing row pass
                 long long in_row = p->M, blk_stride = 0;
                 int lblk = 62;
@@ -1239,6 +1302,7 @@ struct Exec {
 
     fmmfft_status_t run_forward() {
         fmmfft_status_t st;
+        if (p->direct) return mfft();
 #define STEP(stage, call) if ((st = mark(stage))) return st; if ((st = call)) return st;
         STEP(ST_COMM_S, comm_S())
         STEP(ST_NEAR, near_up())
@@ -1319,6 +1383,71 @@ static fmmfft_status_t execute_t(fmmfft_plan_s* p, const void* in, void* out, cu
 using namespace fmmfft;
 
 // ====================================================================== C ABI
+// ---------------------------------------------------------------- autotuner
+static double tune_error(int Q, fmmfft_precision_t prec) {
+    const double trunc = 1.7e-3 * std::pow(6.3, -(double)(Q - 2));      // oracle Q sweep
+    return std::max(trunc, prec == FMMFFT_C64 ? 2.6e-7 : 3e-14);
+}
+
+// roofline model of one execute (seconds), per GPU: HBM passes, S2T flops on the tensor pipe
+// (c64) or FFMA / DFMA, the tree's flops at the register-blocked kernels' measured efficiency,
+// and a per-launch latency
+static double tune_model(long long N, int P, int G, int B, int Q, int M_L, fmmfft_precision_t prec) {
+    const double esz = prec == FMMFFT_C64 ? 8 : 16;
+    const double n = (double)N / G, fmm = (double)(P - 1) / P;
+    const int L = ilog2(N / ((long long)P * M_L));
+    const double hbm = 6.4e12, alu = prec == FMMFFT_C64 ? 74e12 : 37e12;
+    const double tc = prec == FMMFFT_C64 ? 279e12 * 0.25 : 0.0;        // 3xTF32, smem-operand bound
+    const int lM = ilog2(N / P);
+    const int mpass = lM <= 14 ? 1 : (lM <= 22 ? 2 : 3);
+    double t = (2 + 2 + 2 * mpass) * n * esz / hbm;                    // s2m, post_pfft, M-FFT passes
+    if (prec == FMMFFT_C64) t += n * esz / hbm;                         // the S' copy
+    const double s2t = 6.0 * 2 * M_L * fmm * n;
+    t += prec == FMMFFT_C64 && M_L == 64 ? s2t / tc : s2t / (0.35 * alu);
+    const double far = 2.0 * (20.0 * Q * Q / M_L + 4.0 * Q) * fmm * n;
+    t += far / (0.3 * alu) + ((1 << B) * ((1 << B) - 3)) * 4.0 * Q * Q * (P - 1) / (0.05 * alu);
+    const int launches = 6 + 2 * std::max(0, L - B);
+    t += launches * 4e-6;
+    if (G > 1) t += (double)(G - 1) / G * n * esz / 700e9;              // the all-to-all over NVLink
+    return t;
+}
+
+template <typename R>
+static fmmfft_status_t tune_measure(long long N, int P, int B, int Q, int M_L, fmmfft_precision_t prec, float* ms) {
+    fmmfft_plan_t pl = nullptr;
+    fmmfft_status_t st = fmmfft_plan_ex(&pl, N, P, 1, B, Q, prec, M_L, 0u);
+    if (st) return st;
+    void *x = nullptr, *y = nullptr;
+    const size_t bytes = (size_t)N * sizeof(C2<R>);
+    cudaStream_t s = nullptr;
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    cudaError_t e = cudaMalloc(&x, bytes);
+    if (e == cudaSuccess) e = cudaMalloc(&y, bytes);
+    if (e == cudaSuccess) e = cudaMemset(x, 0x3c, bytes);               // finite values (~1e-2 .. 1)
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaEventCreate(&e0);
+    if (e == cudaSuccess) e = cudaEventCreate(&e1);
+    if (e != cudaSuccess) st = fail(FMMFFT_CUDA_ERROR, "autotune scratch: %s", cudaGetErrorString(e));
+    for (int i = 0; i < 3 && !st; ++i) st = fmmfft_execute(pl, x, y, s);
+    if (!st) {
+        cudaEventRecord(e0, s);
+        for (int i = 0; i < 5 && !st; ++i) st = fmmfft_execute(pl, x, y, s);
+        cudaEventRecord(e1, s);
+        e = cudaEventSynchronize(e1);
+        float t = 0;
+        if (e == cudaSuccess) e = cudaEventElapsedTime(&t, e0, e1);
+        if (e != cudaSuccess) st = fail(FMMFFT_CUDA_ERROR, "autotune timing: %s", cudaGetErrorString(e));
+        *ms = t / 5;
+    }
+    if (e0) cudaEventDestroy(e0);
+    if (e1) cudaEventDestroy(e1);
+    if (s) cudaStreamDestroy(s);
+    if (x) cudaFree(x);
+    if (y) cudaFree(y);
+    fmmfft_destroy(pl);
+    return st;
+}
+
 extern "C" {
 
 const char* fmmfft_last_error(void) { return g_last_error.c_str(); }
@@ -1359,13 +1488,52 @@ fmmfft_status_t fmmfft_comm_destroy(void) {
     return FMMFFT_SUCCESS;
 }
 
+// FMMFFT_FLAG_DIRECT: the in-house Cooley-Tukey comparator — the same
+// four-step FFT kernels (k_fft_col + k_fft_rowt) on the whole length-N vector, no FMM.
+static fmmfft_status_t plan_direct(fmmfft_plan_t* plan, long long N, int G, fmmfft_precision_t precision, unsigned flags) {
+    if (!pow2(N)) return fail(FMMFFT_INVALID_VALUE, "N must be a power of two");
+    if (G != 1) return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_DIRECT: single GPU only (G = 1)");
+    if (flags & (FMMFFT_FLAG_VIRTUAL | FMMFFT_FLAG_PROFILE)) return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_DIRECT: no virtual / profile");
+    int dev = 0;
+    CUDA_TRY(cudaGetDevice(&dev));
+    cudaDeviceProp prop;
+    CUDA_TRY(cudaGetDeviceProperties(&prop, dev));
+    if (prop.major != 10 || prop.minor != 0) return fail(FMMFFT_UNSUPPORTED, "sm_100a only");
+    fmmfft_status_t st = precision == FMMFFT_C64 ? init_kernel_attrs<float>() : init_kernel_attrs<double>();
+    if (st) return st;
+    fmmfft_plan_s* p = new fmmfft_plan_s;
+    p->N = N; p->M = N; p->Mg = N; p->P = 1; p->G = 1; p->prec = precision; p->flags = flags; p->device = dev;
+    p->direct = true;
+    p->inverse = (flags & FMMFFT_FLAG_INVERSE) != 0;
+    p->esz = precision == FMMFFT_C64 ? 8 : 16;
+    p->rsz = p->esz / 2;
+    choose_fourstep(p, ilog2(N), precision == FMMFFT_C64 ? 11 : 10);
+    if (!p->fs_lr) { delete p; return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_DIRECT: need 2^10 <= N <= 2^%d", precision == FMMFFT_C64 ? 33 : 30); }
+    const char* g_env = getenv("FMMFFT_NO_GRAPH");
+    p->use_graph = !(g_env && g_env[0] == '1');
+    p->ranks.resize(1);
+    st = dalloc(p, &p->ranks[0].tmp, (size_t)N * p->esz);
+    if (!st && p->inverse) st = dalloc(p, &p->ranks[0].cin, (size_t)N * p->esz);
+    if (!st) {
+        cudaError_t e = cudaStreamCreateWithFlags(&p->cap_stream, cudaStreamNonBlocking);
+        if (e != cudaSuccess) st = fail(FMMFFT_CUDA_ERROR, "stream setup: %s", cudaGetErrorString(e));
+    }
+    if (st) { destroy_plan(p); return st; }
+    *plan = p;
+    return FMMFFT_SUCCESS;
+}
+
 fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, int B, int Q,
                                fmmfft_precision_t precision, int M_L, unsigned flags) {
     if (!plan) return fail(FMMFFT_INVALID_VALUE, "plan is NULL");
     *plan = nullptr;
     if (precision != FMMFFT_C64 && precision != FMMFFT_C128) return fail(FMMFFT_INVALID_VALUE, "bad precision");
+    if (flags & FMMFFT_FLAG_DIRECT) return plan_direct(plan, N, G, precision, flags);
+    if (precision != FMMFFT_C64 && precision != FMMFFT_C128) return fail(FMMFFT_INVALID_VALUE, "bad precision");
     if (!pow2(N) || !pow2(P) || !pow2(M_L)) return fail(FMMFFT_INVALID_VALUE, "N, P, M_L must be powers of two");
-    if (P < 2 || P > 2048) return fail(FMMFFT_INVALID_VALUE, "need 2 <= P <= 2048 (P=%d)", P);
+    // k_post_pfft holds >= 8 m-rows of all P points in one CTA's shared memory tile
+    const int Pmax = precision == FMMFFT_C64 ? 1024 : 512;
+    if (P < 2 || P > Pmax) return fail(FMMFFT_INVALID_VALUE, "need 2 <= P <= %d (P=%d)", Pmax, P);
     if (!(G == 1 || G == 2 || G == 4 || G == 8)) return fail(FMMFFT_INVALID_VALUE, "G must be 1, 2, 4 or 8");
     if (P % G) return fail(FMMFFT_INVALID_VALUE, "P %% G != 0");
     if (M_L < 16 || M_L > 128) return fail(FMMFFT_INVALID_VALUE, "need 16 <= M_L <= 128");
@@ -1427,6 +1595,7 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
     p->s2t_tc = precision == FMMFFT_C64 && M_L == 64 && (p->nb % S2TC_BOXES) == 0;
     if (const char* e = getenv("FMMFFT_S2T")) p->s2t_tc = p->s2t_tc && e[0] == 't';
     if (const char* e = getenv("FMMFFT_DOWN")) p->lvl_off = e[0] == 't';
+    if (const char* e = getenv("FMMFFT_PP")) p->pp_old = e[0] == 't';
     if (const char* e = getenv("FMMFFT_S2M_NBX")) p->s2m_nbx = atoi(e) == 1 ? 1 : 2;
     if (const char* e = getenv("FMMFFT_S2M_PC")) { const int v = atoi(e); if (v == 8 || v == 16 || (v == 32 && precision == FMMFFT_C64)) p->s2m_pc = v; }
     if (const char* e = getenv("FMMFFT_PP_MS")) { const int v = atoi(e); if (v >= 8 && v <= M_L && pow2(v)) p->pp_ms = v; }
@@ -1448,24 +1617,15 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
     }
     {   // rows longer than one CTA's shared memory: the four-step passes (FMMFFT_MFFT=pass keeps k_fft_pass)
         const int lM = ilog2(p->M);
-        const int mx = precision == FMMFFT_C64 ? 11 : 10;
+        int mx = 10;                     // 11-bit passes (1 CTA per SM) measured slower than 3 passes of <= 10 bits
+        if (const char* b = getenv("FMMFFT_FS_MAXBITS")) mx = std::max(6, std::min(mx, atoi(b)));
         const char* e = getenv("FMMFFT_MFFT");
         const bool want = !(e && e[0] == 'p') && !(getenv("FMMFFT_ROWFFT") && getenv("FMMFFT_ROWFFT")[0] == '0');
         // FMMFFT_MFFT=fs forces it; by default also rows of >= 2^13 points when there are fewer rows
         // than SMs (k_fft_row would run one CTA per row on part of the GPU)
         const bool few_rows = P / G < 148 && lM >= 13 && !getenv("FMMFFT_ROWFFT_CL") && !(e && e[0] == 'r');
         if (want && ((e && e[0] == 'f' && lM >= 10) || few_rows)) { p->row_fft1 = false; p->row_cl = 0; }
-        if (want && !p->row_fft1 && !p->row_cl && lM >= 10 && lM <= 3 * mx) {
-            if (lM <= 2 * mx) {
-                p->fs_lr = std::min(mx, (lM + 1) / 2);
-                p->fs_lc1 = lM - p->fs_lr;
-            } else {
-                p->fs_lr = std::min(mx, (lM + 2) / 3);
-                p->fs_lc1 = std::min(mx, (lM - p->fs_lr + 1) / 2);
-                p->fs_lc2 = lM - p->fs_lr - p->fs_lc1;
-            }
-            if (p->fs_lc1 < 5 || p->fs_lr < 5 || (p->fs_lc2 && p->fs_lc2 < 5)) p->fs_lr = p->fs_lc1 = p->fs_lc2 = 0;
-        }
+        if (want && !p->row_fft1 && !p->row_cl) choose_fourstep(p, lM, mx);
     }
     st = precision == FMMFFT_C64 ? build_tables<float>(p) : build_tables<double>(p);
     if (!st) {
@@ -1504,6 +1664,44 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
     }
     if (st) { destroy_plan(p); return st; }
     *plan = p;
+    return FMMFFT_SUCCESS;
+}
+
+fmmfft_status_t fmmfft_autotune(long long N, int G, fmmfft_precision_t precision, double tol, int measure, fmmfft_tune_t* best) {
+    if (!best) return fail(FMMFFT_INVALID_VALUE, "best is NULL");
+    if (precision != FMMFFT_C64 && precision != FMMFFT_C128) return fail(FMMFFT_INVALID_VALUE, "bad precision");
+    if (!pow2(N) || !(G == 1 || G == 2 || G == 4 || G == 8)) return fail(FMMFFT_INVALID_VALUE, "N a power of two, G in {1,2,4,8}");
+    if (measure && G != 1) return fail(FMMFFT_INVALID_VALUE, "measured autotuning is single-GPU (G = 1); use the model for G > 1");
+    int Q = 0;
+    for (int q : {8, 16, 24})
+        if (tune_error(q, precision) * 4 <= tol) { Q = q; break; }
+    if (!Q) return fail(FMMFFT_INVALID_VALUE, "no Q in {8,16,24} reaches tol=%g at this precision", tol);
+    const int M_L = 64;
+    *best = fmmfft_tune_t{0, 0, Q, M_L, 0.f, tune_error(Q, precision), 0};
+    double best_t = 1e30;
+    for (int P = std::max(2, G); P <= (precision == FMMFFT_C64 ? 1024 : 512); P *= 2) {
+        if (P % G || N % ((long long)P * M_L)) continue;
+        const long long nleaf = N / ((long long)P * M_L);
+        if (nleaf % G) continue;
+        const int L = ilog2(nleaf);
+        for (int B = 2; B <= 4; ++B) {
+            if (L < B) continue;
+            double t;
+            if (measure) {
+                float ms = 0;
+                const fmmfft_status_t st = precision == FMMFFT_C64 ? tune_measure<float>(N, P, B, Q, M_L, precision, &ms)
+                                                                   : tune_measure<double>(N, P, B, Q, M_L, precision, &ms);
+                if (st == FMMFFT_UNSUPPORTED || st == FMMFFT_INVALID_VALUE) continue;   // not a valid plan here
+                if (st) return st;
+                t = ms * 1e-3;
+            } else {
+                t = tune_model(N, P, G, B, Q, M_L, precision);
+            }
+            ++best->candidates;
+            if (t < best_t) { best_t = t; best->P = P; best->B = B; best->ms = (float)(t * 1e3); }
+        }
+    }
+    if (!best->P) return fail(FMMFFT_INVALID_VALUE, "no valid (P, B) for N=%lld, G=%d with M_L=64", N, G);
     return FMMFFT_SUCCESS;
 }
 

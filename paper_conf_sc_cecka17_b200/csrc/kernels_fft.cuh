@@ -731,4 +731,93 @@ k_conj_scale(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, long long n,
     }
 }
 
+// ---------------------------------------------------------------------------------------------
+// k_post_pfft_r: the same L2T + POST + P-point FFT + transposed store for P <= 32 with the whole
+// P-point column of one m in one thread's registers (no shared-memory FFT tile, no barriers in
+// the FFT): thread (box b, m) loads T_near[p][b][.][m] for all p (coalesced over m), adds
+// L2T_{mq} L^L_{pqb} (L^L of its box broadcast from shared memory, two p per 16-byte load),
+// applies POST, runs the P-point DFT in registers (radix 2/4/8/16, 32 = 2 x 16) and stores
+// W[k2][b M_L + m] for every k2 (coalesced over m). CTA = NBX consecutive boxes x M_L threads.
+// ---------------------------------------------------------------------------------------------
+template <typename R, int LP, int QT>
+__global__ void __launch_bounds__(256)
+k_post_pfft_r(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2<R>* __restrict__ r,
+              const C2<R>* __restrict__ rho, const R* __restrict__ s2m, C2<R>* __restrict__ W, int lML, int Mg) {
+    pdl_trigger();
+    using C = C2<R>;
+    constexpr int P = 1 << LP, Q = QT;
+    const int M_L = 1 << lML;
+    const int nbx = blockDim.x >> lML;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    C* Lsm = reinterpret_cast<C*>(smem_raw);                      // [nbx][Q][P]
+    C* rr = Lsm + nbx * Q * P;                                     // [P] r_p
+    C* rh = rr + P;                                                // [P] rho_p
+    C* tw32 = rh + P;                                              // [16] w_32^k
+    const int tid = threadIdx.x, bx = tid >> lML, m = tid & (M_L - 1);
+    const int b = blockIdx.x * nbx + bx;
+    R w[Q];                                                        // L2T_{mq} = S2M_{qm}
+#pragma unroll
+    for (int q = 0; q < Q; ++q) w[q] = __ldg(s2m + (size_t)q * M_L + m);
+    if (tid < 16) tw32[tid] = twiddle_pow2(R(0), tid, 5);
+    pdl_wait();                                                   // T_near / L^L / r from the FMM stages
+    {
+        constexpr int V = 16 / sizeof(C);
+        const C* src = LL + (size_t)blockIdx.x * nbx * Q * P;
+        for (int idx = tid; idx < nbx * Q * P / V; idx += blockDim.x) cp_async<16>(Lsm + idx * V, src + idx * V);
+        if (tid < P) { rr[tid] = ldg_c(r + tid); rh[tid] = ldg_c(rho + tid); }
+    }
+    C v[P];
+    const R* tn = reinterpret_cast<const R*>(Tn) + ((size_t)b << (lML + 1)) + m;
+#pragma unroll
+    for (int p = 0; p < P; ++p) {
+        v[p].x = __ldg(tn + (size_t)p * 2 * Mg);
+        v[p].y = __ldg(tn + (size_t)p * 2 * Mg + M_L);
+    }
+    cp_async_wait_all();
+    __syncthreads();
+    const C* Lb = Lsm + bx * Q * P;
+#pragma unroll
+    for (int p = 0; p < P; p += 2) {
+        C a0 = zero<C>(), a1 = zero<C>();
+#pragma unroll
+        for (int q = 0; q < Q; ++q) {
+            C l0, l1;
+            if constexpr (sizeof(R) == 4) {
+                const float4 l = *reinterpret_cast<const float4*>(Lb + q * P + p);
+                l0 = make_float2(l.x, l.y); l1 = make_float2(l.z, l.w);
+            } else {
+                l0 = Lb[q * P + p]; l1 = Lb[q * P + p + 1];
+            }
+            rfma(a0, w[q], l0);
+            rfma(a1, w[q], l1);
+        }
+        if (p > 0) {                                               // C_0 = I (R1)
+            C t = cadd(v[p], a0);
+            t.x -= rr[p].y; t.y += rr[p].x;                        // + i r_p
+            v[p] = cmul(rh[p], t);
+        }
+        C t = cadd(v[p + 1], a1);
+        t.x -= rr[p + 1].y; t.y += rr[p + 1].x;
+        v[p + 1] = cmul(rh[p + 1], t);
+    }
+    // P-point DFT over p, natural order
+    if constexpr (P <= 16) {
+        dft_small<P>(v);
+    } else {                                                      // 32 = 2 x 16: X[k] = E[k] + w^k O[k]
+        C e[16], o[16];
+#pragma unroll
+        for (int t = 0; t < 16; ++t) { e[t] = v[2 * t]; o[t] = v[2 * t + 1]; }
+        dft16(e); dft16(o);
+#pragma unroll
+        for (int k = 0; k < 16; ++k) {
+            const C ow = cmul(o[k], tw32[k]);
+            v[k] = cadd(e[k], ow);
+            v[k + 16] = csub(e[k], ow);
+        }
+    }
+    C* dst = W + ((size_t)b << lML) + m;
+#pragma unroll
+    for (int k2 = 0; k2 < P; ++k2) dst[(size_t)k2 * Mg] = v[k2];
+}
+
 }  // namespace fmmfft

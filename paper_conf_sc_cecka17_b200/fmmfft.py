@@ -15,7 +15,7 @@ import ctypes
 import torch
 
 from . import _lib
-from ._lib import C64, C128, FLAG_DEBUG, FLAG_INVERSE, FLAG_PROFILE, FLAG_VIRTUAL, check, lib
+from ._lib import C64, C128, FLAG_DEBUG, FLAG_DIRECT, FLAG_INVERSE, FLAG_PROFILE, FLAG_VIRTUAL, check, lib
 
 _DT = {"c64": (C64, torch.complex64), "c128": (C128, torch.complex128)}
 
@@ -41,6 +41,15 @@ def init_comm(group=None) -> None:
     check(lib.fmmfft_comm_init(rank, world, bytes(buf.cpu().numpy().tobytes())))
 
 
+def autotune(N: int, G: int = 1, precision: str = "c64", tol: float = 1e-5, measure: bool = True) -> dict:
+    """(P, B, Q, M_L) for an FMM-FFT of length N on G GPUs meeting relative-l2 error `tol`
+    (fmmfft_autotune: Q from the error model, (P, B) timed on the current device when measure,
+    else ranked by the roofline model). Returns the plan arguments plus ms / error / candidates."""
+    t = _lib.Tune()
+    check(lib.fmmfft_autotune(N, G, _DT[precision][0], float(tol), 1 if measure else 0, ctypes.byref(t)))
+    return {f: getattr(t, f) for f, _ in _lib.Tune._fields_}
+
+
 def destroy_comm() -> None:
     check(lib.fmmfft_comm_destroy())
 
@@ -59,13 +68,15 @@ class _DevView:
 class FmmFFT:
     def __init__(self, N: int, P: int, G: int = 1, B: int = 2, Q: int = 16, precision: str = "c64",
                  M_L: int = 64, virtual: bool = False, profile: bool = False, debug: bool = False,
-                 inverse: bool = False):
+                 inverse: bool = False, direct: bool = False):
+        """direct=True: no FMM — the plain four-step FFT of length N on one GPU with the same M-FFT
+        kernels (the in-house Cooley-Tukey comparator; P, B, Q, M_L ignored)."""
         self.N, self.P, self.G, self.B, self.Q, self.M_L = N, P, G, B, Q, M_L
         self.precision = precision
         self.virtual = virtual
         self._prec, self.dtype = _DT[precision]
         flags = (FLAG_VIRTUAL if virtual else 0) | (FLAG_PROFILE if profile else 0) | (FLAG_DEBUG if debug else 0) | \
-                (FLAG_INVERSE if inverse else 0)
+                (FLAG_INVERSE if inverse else 0) | (FLAG_DIRECT if direct else 0)
         self.inverse = inverse
         h = ctypes.c_void_p()
         check(lib.fmmfft_plan_ex(ctypes.byref(h), N, P, G, B, Q, self._prec, M_L, flags))

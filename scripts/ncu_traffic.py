@@ -32,7 +32,7 @@ def load(rep):
     for r in rows[2:]:
         if len(r) != len(hdr):
             continue
-        d = {"kernel": r[hdr.index("Kernel Name")].split("(")[0].replace("void ", "").strip()}
+        d = {"kernel": r[hdr.index("Kernel Name")].split("(")[0].replace("void ", "").replace("fmmfft::", "").strip()}
         for m in METRICS:
             if m not in hdr:
                 continue

@@ -82,3 +82,19 @@ def test_package_has_no_cpu_fallback():
             src = open(os.path.join(pkg, f)).read()
             assert "oracle" not in src.replace("oracle/", ""), f
             assert "numpy.fft" not in src and "np.fft" not in src and "torch.fft" not in src, f
+
+
+# ------------------------------------------------------------------ autotuner model mode (host only)
+def test_autotune_model_host_only():
+    from paper_conf_sc_cecka17_b200 import autotune
+    from paper_conf_sc_cecka17_b200._lib import FmmfftError
+    t = autotune(1 << 26, G=8, precision="c64", tol=1e-5, measure=False)
+    assert t["Q"] == 8 and t["M_L"] == 64 and t["P"] % 8 == 0 and 2 <= t["B"] <= 4
+    L = (26 - (t["P"].bit_length() - 1) - 6)
+    assert L >= t["B"] and (1 << L) % 8 == 0 and t["candidates"] > 3 and t["error"] * 4 <= 1e-5
+    t = autotune(1 << 28, G=8, precision="c128", tol=1e-11, measure=False)
+    assert t["Q"] == 16
+    with pytest.raises(FmmfftError):
+        autotune(1 << 20, precision="c64", tol=1e-8, measure=False)      # below the fp32 floor
+    with pytest.raises(FmmfftError):
+        autotune(1 << 20, G=2, precision="c64", measure=True)           # measuring is G = 1 only

@@ -287,3 +287,43 @@ def test_inverse_vs_oracle(F, N, P, B, Q, prec, M_L, G):
     fwd = F(N=N, P=P, G=G, B=B, Q=Q, precision=prec, M_L=M_L, virtual=G > 1)
     z = inv(fwd(torch.from_numpy(x).cuda())).cpu().numpy()
     assert rel(z, x) < 2 * TOL_E2E[prec]
+
+
+# ------------------------------------------------------------------ in-house four-step FFT, no FMM (§8(f) NEXT-3)
+@pytest.mark.parametrize("N,prec,inverse", [
+    (1 << 13, "c64", False), (1 << 20, "c64", False), (1 << 23, "c64", False),   # 2 / 2 / 3 passes
+    (1 << 21, "c128", False), (1 << 16, "c128", True), (1 << 22, "c64", True),
+])
+def test_direct_fft(F, N, prec, inverse):
+    x = SI.complex_uniform(0, N, dtype=NPDT[prec])
+    plan = F(N=N, P=1, precision=prec, direct=True, inverse=inverse)
+    y = plan(torch.from_numpy(x).cuda()).cpu().numpy()
+    ref = O.fft_radix2(x, inverse=inverse)
+    assert rel(y, ref) < (1e-6 if prec == "c64" else 1e-13)
+
+
+def test_direct_rejects_multi_gpu(F):
+    from paper_conf_sc_cecka17_b200._lib import FmmfftError
+    with pytest.raises(FmmfftError):
+        F(N=1 << 20, P=2, G=2, virtual=True, direct=True)
+
+
+# ------------------------------------------------------------------ autotuner, measured (§8(f) NEXT-2)
+def test_autotune_measured_meets_tol(F):
+    from paper_conf_sc_cecka17_b200 import autotune
+    N = 1 << 20
+    t = autotune(N, G=1, precision="c64", tol=1e-5, measure=True)
+    assert t["candidates"] >= 3 and t["ms"] > 0
+    plan, x, y = run(F, N, t["P"], t["B"], t["Q"], "c64", t["M_L"])
+    assert rel(y, O.fft_radix2(x)) < 1e-5
+
+
+@pytest.mark.parametrize("env", [None, {"FMMFFT_PP": "tile"}])
+@pytest.mark.parametrize("P,Q,prec", [(16, 16, "c64"), (32, 8, "c64"), (8, 24, "c128"), (2, 16, "c64")])
+def test_post_pfft_variants(F, monkeypatch, env, P, Q, prec):
+    """k_post_pfft_r (P <= 32, registers) and the shared-memory-tile k_post_pfft agree with the oracle."""
+    for k, v in (env or {}).items():
+        monkeypatch.setenv(k, v)
+    N = 1 << 18
+    plan, x, y = run(F, N, P, 2, Q, prec, 64)
+    assert rel(y, O.fft_radix2(x)) < (1e-5 if prec == "c64" else 1e-11)
