@@ -396,11 +396,11 @@ def run_fmmfft(args, rank, world, local_rank):
         dist.all_reduce(nx)
     parseval = float(ny / (N * nx) - 1)
 
-    cufft_comp = cufft_comparator(x, flush, min(args.steps, 50)) if world == 1 else None
+    cufft_comp = cufft_comparator(x, flush, min(args.steps, 50)) if world == 1 and not args.no_extras else None
     # context: the library's own autotuner on the same N, precision and
     # error bound — (P, B, Q) free instead of the config's — timed the same way
     autotuned = None
-    if world == 1:
+    if world == 1 and not args.no_extras:
         try:
             from paper_conf_sc_cecka17_b200 import autotune
             tol = 1e-5 if prec == "c64" else 1e-11
@@ -493,6 +493,8 @@ def main():
     ap.add_argument("--impl", default="fmmfft", choices=["fmmfft", "reference"])
     ap.add_argument("--workload", default=None, choices=sorted(WORKLOADS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-extras", action="store_true",
+                    help="skip the comparators and the autotuner pick (profiling runs: only the FMM-FFT's launches)")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     rank = int(os.environ.get("RANK", "0"))

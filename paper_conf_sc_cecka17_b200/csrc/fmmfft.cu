@@ -213,7 +213,9 @@ struct fmmfft_plan_s {
     int fs_lc1 = 0, fs_lc2 = 0, fs_lr = 0;   // four-step large-M FFT: column pass bits (2nd: 0 = none), row pass bits
     int s2m_nbx = 0, s2m_pc = 0, pp_ms = 0;  // tuning knobs (FMMFFT_S2M_NBX, FMMFFT_S2M_PC, FMMFFT_PP_MS); 0 = default
     bool inverse = false;            // FMMFFT_FLAG_INVERSE: x = F_N^{-1} y
-    bool pp_old = false;             // FMMFFT_PP=tile: the shared-memory-tile k_post_pfft for every P
+    bool pp_old = false;
+    bool fs_narrow = false;
+    int s2t_tpc = 0;                 // FMMFFT_S2T_TPC: tiles per k_s2t_tc CTA (0 = one wave)          // FMMFFT_FS_NARROW=1: 11-bit (c64) / 10-bit (c128) four-step passes on 4-column CTAs             // FMMFFT_PP=tile: the shared-memory-tile k_post_pfft for every P
     bool direct = false;             // FMMFFT_FLAG_DIRECT: plain four-step FFT of length N, no FMM
     bool lvl_off = false;            // FMMFFT_DOWN=tree: every down level in k_tree_down (no k_m2l_lvl)
     bool s2t_tc = false;             // S2T on tcgen05 (k_s2t_tc): complex64, M_L = 64, nb % 128 == 0
@@ -519,6 +521,9 @@ static fmmfft_status_t init_kernel_attrs() {
         }
         if constexpr (sizeof(R) == 4) set((const void*)k_s2t_tc);
         set((const void*)k_base_sg<R, 4, sizeof(R) == 4 ? 8 : 4, 4>);
+        set((const void*)k_post_pfft_r2<R, 8>);
+        set((const void*)k_post_pfft_r2<R, 16>);
+        set((const void*)k_post_pfft_r2<R, 24>);
         for (int lp = 1; lp <= 5; ++lp)
             dispatch<1, 2, 3, 4, 5>(lp, [&](auto v) {
                 set((const void*)k_post_pfft_r<R, decltype(v)::value, 8>);
@@ -558,6 +563,10 @@ static fmmfft_status_t init_kernel_attrs() {
                 if constexpr (LV <= fs_max<R>()) {
                     set((const void*)k_fft_col<R, LV, fs_cols<R>(LV)>);
                     set((const void*)k_fft_rowt<R, LV, fs_cols<R>(LV)>);
+                    if constexpr (LV >= fs_max<R>() - 1) {
+                        set((const void*)k_fft_col<R, LV, 4>);
+                        set((const void*)k_fft_rowt<R, LV, 4>);
+                    }
                 }
             });
         for (int ll = 8; ll <= kRowFftMax<R>; ++ll)
@@ -689,7 +698,8 @@ struct Exec {
                 // tiles per CTA: the fewest that keep the grid within one wave of 148 SMs
                 // (one CTA per SM: TMEM + ~180 KB of shared memory)
                 const int cpp = std::max(1, 148 / (p->P - 1));             // CTAs per p
-                const int tpc = (ntile + cpp - 1) / cpp;
+                int tpc = (ntile + cpp - 1) / cpp;
+                if (p->s2t_tpc) tpc = std::min(ntile, p->s2t_tpc);
                 for (RankBufs& rb : p->ranks) {
                     const dim3 grid((unsigned)((ntile + tpc - 1) / tpc), (unsigned)(p->P - 1));
                     launch_pdl(k_s2t_tc, grid, S2TC_THREADS, s2tc_smem_bytes(), p->side, (const C*)rb.Sp, (const C*)rb.haloL,
@@ -1099,6 +1109,22 @@ struct Exec {
 
     // ---- L2T + POST + P-FFT
     fmmfft_status_t post_pfft() {
+        // P = 64: two threads per (box, m), registers + one shuffle exchange (k_post_pfft_r2)
+        if (p->P == 64 && (p->Q == 8 || p->Q == 16 || p->Q == 24) && p->M_L <= 128 && !p->pp_old) {
+            const int nbx = std::max(1, std::min(p->nb, 128 / p->M_L));
+            if (p->nb % nbx == 0) {
+                const size_t smem = ((size_t)nbx * p->Q * 64 + 2 * 64 + 48) * sizeof(C);
+                for (RankBufs& rb : p->ranks) {
+                    dispatch<8, 16, 24>(p->Q, [&](auto qv) {
+                        launch_pdl(k_post_pfft_r2<R, decltype(qv)::value>, (unsigned)(p->nb / nbx), 2 * nbx * p->M_L, smem, s,
+                                   (const C*)rb.Tn, (const C*)rb.Lloc[p->L], (const C*)rb.r, (const C*)p->rho,
+                                   (const R*)p->s2m, (C*)rb.W, ilog2(p->M_L), (int)p->Mg);
+                    });
+                    LAUNCH_CHECK();
+                }
+                return FMMFFT_SUCCESS;
+            }
+        }
         // P <= 32 (and a specialised Q): the register-resident variant, one thread per (box, m)
         if (p->P <= 32 && p->P >= 2 && (p->Q == 8 || p->Q == 16 || p->Q == 24) && p->M_L <= 256 && !p->pp_old) {
             const int nbx = std::max(1, std::min(p->nb, 256 / p->M_L));
@@ -1174,9 +1200,17 @@ struct Exec {
         bool ok = dispatch<5, 6, 7, 8, 9, 10, 11>(LCv, [&](auto lc) {
             constexpr int LC = decltype(lc)::value;
             constexpr int CB = fs_cols<R>(LC);
-            if constexpr (LC <= fs_max<R>())
+            if constexpr (LC <= fs_max<R>()) {
+                if constexpr (LC >= fs_max<R>() - 1) {
+                    if (p->fs_narrow) {             // 4 columns (32-byte runs): ~70 KB, several CTAs per SM
+                        launch_pdl(k_fft_col<R, LC, 4>, dim3((unsigned)((1LL << lMi) / 4), (unsigned)nseq), 4 << (LC - 4),
+                                   fft_col_smem<R, LC, 4>(), s, in_, out_, lMs, lMi, lSdiv, (long long)p->M, in_row, lblk, blk_stride);
+                        return;
+                    }
+                }
                 launch_pdl(k_fft_col<R, LC, CB>, dim3((unsigned)((1LL << lMi) / CB), (unsigned)nseq), CB << (LC - 4),
                            fft_col_smem<R, LC, CB>(), s, in_, out_, lMs, lMi, lSdiv, (long long)p->M, in_row, lblk, blk_stride);
+            }
         });
         if (!ok) return fail(FMMFFT_UNSUPPORTED, "k_fft_col: 2^%d", LCv);
         LAUNCH_CHECK();
@@ -1210,9 +1244,17 @@ struct Exec {
                 bool ok = dispatch<5, 6, 7, 8, 9, 10, 11>(p->fs_lr, [&](auto ll) {
                     constexpr int LL = decltype(ll)::value;
                     constexpr int CR = fs_cols<R>(LL);
-                    if constexpr (LL <= fs_max<R>())
+                    if constexpr (LL <= fs_max<R>()) {
+                        if constexpr (LL >= fs_max<R>() - 1) {
+                            if (p->fs_narrow) {
+                                launch_pdl(k_fft_rowt<R, LL, 4>, (unsigned)(trows / 4), 4 << (LL - 4), fft_rowt_smem<R, LL, 4>(), s,
+                                           bsrc, dst, (long long)p->M, lrpr);
+                                return;
+                            }
+                        }
                         launch_pdl(k_fft_rowt<R, LL, CR>, (unsigned)(trows / CR), CR << (LL - 4), fft_rowt_smem<R, LL, CR>(), s,
                                    bsrc, dst, (long long)p->M, lrpr);
+                    }
                 });
                 if (!ok) return fail(FMMFFT_UNSUPPORTED, "k_fft_rowt: 2^%d", p->fs_lr);
                 LAUNCH_CHECK();
@@ -1596,6 +1638,7 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
     if (const char* e = getenv("FMMFFT_S2T")) p->s2t_tc = p->s2t_tc && e[0] == 't';
     if (const char* e = getenv("FMMFFT_DOWN")) p->lvl_off = e[0] == 't';
     if (const char* e = getenv("FMMFFT_PP")) p->pp_old = e[0] == 't';
+    if (const char* e = getenv("FMMFFT_S2T_TPC")) p->s2t_tpc = std::max(0, atoi(e));
     if (const char* e = getenv("FMMFFT_S2M_NBX")) p->s2m_nbx = atoi(e) == 1 ? 1 : 2;
     if (const char* e = getenv("FMMFFT_S2M_PC")) { const int v = atoi(e); if (v == 8 || v == 16 || (v == 32 && precision == FMMFFT_C64)) p->s2m_pc = v; }
     if (const char* e = getenv("FMMFFT_PP_MS")) { const int v = atoi(e); if (v >= 8 && v <= M_L && pow2(v)) p->pp_ms = v; }
@@ -1618,6 +1661,8 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
     {   // rows longer than one CTA's shared memory: the four-step passes (FMMFFT_MFFT=pass keeps k_fft_pass)
         const int lM = ilog2(p->M);
         int mx = 10;                     // 11-bit passes (1 CTA per SM) measured slower than 3 passes of <= 10 bits
+        if (const char* nw = getenv("FMMFFT_FS_NARROW")) p->fs_narrow = nw[0] == '1';
+        if (p->fs_narrow) mx = precision == FMMFFT_C64 ? 11 : 10;
         if (const char* b = getenv("FMMFFT_FS_MAXBITS")) mx = std::max(6, std::min(mx, atoi(b)));
         const char* e = getenv("FMMFFT_MFFT");
         const bool want = !(e && e[0] == 'p') && !(getenv("FMMFFT_ROWFFT") && getenv("FMMFFT_ROWFFT")[0] == '0');

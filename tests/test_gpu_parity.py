@@ -319,7 +319,7 @@ def test_autotune_measured_meets_tol(F):
 
 
 @pytest.mark.parametrize("env", [None, {"FMMFFT_PP": "tile"}])
-@pytest.mark.parametrize("P,Q,prec", [(16, 16, "c64"), (32, 8, "c64"), (8, 24, "c128"), (2, 16, "c64")])
+@pytest.mark.parametrize("P,Q,prec", [(16, 16, "c64"), (32, 8, "c64"), (8, 24, "c128"), (2, 16, "c64"), (64, 16, "c64"), (64, 24, "c128")])
 def test_post_pfft_variants(F, monkeypatch, env, P, Q, prec):
     """k_post_pfft_r (P <= 32, registers) and the shared-memory-tile k_post_pfft agree with the oracle."""
     for k, v in (env or {}).items():
