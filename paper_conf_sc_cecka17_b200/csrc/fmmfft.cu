@@ -521,9 +521,6 @@ static fmmfft_status_t init_kernel_attrs() {
         }
         if constexpr (sizeof(R) == 4) set((const void*)k_s2t_tc);
         set((const void*)k_base_sg<R, 4, sizeof(R) == 4 ? 8 : 4, 4>);
-        set((const void*)k_post_pfft_r2<R, 8>);
-        set((const void*)k_post_pfft_r2<R, 16>);
-        set((const void*)k_post_pfft_r2<R, 24>);
         for (int lp = 1; lp <= 5; ++lp)
             dispatch<1, 2, 3, 4, 5>(lp, [&](auto v) {
                 set((const void*)k_post_pfft_r<R, decltype(v)::value, 8>);
@@ -1109,22 +1106,6 @@ struct Exec {
 
     // ---- L2T + POST + P-FFT
     fmmfft_status_t post_pfft() {
-        // P = 64: two threads per (box, m), registers + one shuffle exchange (k_post_pfft_r2)
-        if (p->P == 64 && (p->Q == 8 || p->Q == 16 || p->Q == 24) && p->M_L <= 128 && !p->pp_old) {
-            const int nbx = std::max(1, std::min(p->nb, 128 / p->M_L));
-            if (p->nb % nbx == 0) {
-                const size_t smem = ((size_t)nbx * p->Q * 64 + 2 * 64 + 48) * sizeof(C);
-                for (RankBufs& rb : p->ranks) {
-                    dispatch<8, 16, 24>(p->Q, [&](auto qv) {
-                        launch_pdl(k_post_pfft_r2<R, decltype(qv)::value>, (unsigned)(p->nb / nbx), 2 * nbx * p->M_L, smem, s,
-                                   (const C*)rb.Tn, (const C*)rb.Lloc[p->L], (const C*)rb.r, (const C*)p->rho,
-                                   (const R*)p->s2m, (C*)rb.W, ilog2(p->M_L), (int)p->Mg);
-                    });
-                    LAUNCH_CHECK();
-                }
-                return FMMFFT_SUCCESS;
-            }
-        }
         // P <= 32 (and a specialised Q): the register-resident variant, one thread per (box, m)
         if (p->P <= 32 && p->P >= 2 && (p->Q == 8 || p->Q == 16 || p->Q == 24) && p->M_L <= 256 && !p->pp_old) {
             const int nbx = std::max(1, std::min(p->nb, 256 / p->M_L));

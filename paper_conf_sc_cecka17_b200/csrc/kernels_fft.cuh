@@ -820,109 +820,4 @@ k_post_pfft_r(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const 
     for (int k2 = 0; k2 < P; ++k2) dst[(size_t)k2 * Mg] = v[k2];
 }
 
-// ---------------------------------------------------------------------------------------------
-// k_post_pfft_r2: P = 64 with a PAIR of threads per (box, m) — thread h holds p in [32h, 32h + 32)
-// in registers (L2T + POST for its own p, 16-byte L^L loads), then a decimation-in-frequency
-// split over the pair: after one exchange of 32 values through warp shuffles,
-//   h = 0: X[2k]   = DFT32_k(x[p] + x[p + 32]),
-//   h = 1: X[2k+1] = DFT32_k((x[p] - x[p + 32]) w_64^p),
-// and each thread stores its 32 outputs W[2k + h][b M_L + m]. Lanes are (m, h) pairs, so loads
-// and stores move 64-byte runs of m.
-// ---------------------------------------------------------------------------------------------
-template <typename C> __device__ __forceinline__ C shfl_xor_c(C v, int mask);
-template <> __device__ __forceinline__ float2 shfl_xor_c<float2>(float2 v, int mask) {
-    return make_float2(__shfl_xor_sync(0xffffffffu, v.x, mask), __shfl_xor_sync(0xffffffffu, v.y, mask));
-}
-template <> __device__ __forceinline__ double2 shfl_xor_c<double2>(double2 v, int mask) {
-    return make_double2(__shfl_xor_sync(0xffffffffu, v.x, mask), __shfl_xor_sync(0xffffffffu, v.y, mask));
-}
-
-template <typename R, int QT>
-__global__ void __launch_bounds__(256)
-k_post_pfft_r2(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2<R>* __restrict__ r,
-               const C2<R>* __restrict__ rho, const R* __restrict__ s2m, C2<R>* __restrict__ W, int lML, int Mg) {
-    pdl_trigger();
-    using C = C2<R>;
-    constexpr int P = 64, H = 32, Q = QT;
-    const int M_L = 1 << lML;
-    const int nbx = blockDim.x >> (lML + 1);
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    C* Lsm = reinterpret_cast<C*>(smem_raw);                      // [nbx][Q][P]
-    C* rr = Lsm + nbx * Q * P;                                     // [P] r_p
-    C* rh = rr + P;                                                // [P] rho_p
-    C* tw = rh + P;                                                // [32] w_64^p, then [16] w_32^k
-    const int tid = threadIdx.x, h = tid & 1, mm = tid >> 1;
-    const int bx = mm >> lML, m = mm & (M_L - 1);
-    const int b = blockIdx.x * nbx + bx;
-    R w[Q];
-#pragma unroll
-    for (int q = 0; q < Q; ++q) w[q] = __ldg(s2m + (size_t)q * M_L + m);
-    if (tid < 32) tw[tid] = twiddle_pow2(R(0), tid, 6);
-    else if (tid < 48) tw[tid] = twiddle_pow2(R(0), tid - 32, 5);
-    pdl_wait();
-    {
-        constexpr int V = 16 / sizeof(C);
-        const C* src = LL + (size_t)blockIdx.x * nbx * Q * P;
-        for (int idx = tid; idx < nbx * Q * P / V; idx += blockDim.x) cp_async<16>(Lsm + idx * V, src + idx * V);
-        if (tid < P) { rr[tid] = ldg_c(r + tid); rh[tid] = ldg_c(rho + tid); }
-    }
-    C v[H];
-    const int p0 = h * H;
-    const R* tn = reinterpret_cast<const R*>(Tn) + ((size_t)b << (lML + 1)) + m;
-#pragma unroll
-    for (int t = 0; t < H; ++t) {
-        v[t].x = __ldg(tn + (size_t)(p0 + t) * 2 * Mg);
-        v[t].y = __ldg(tn + (size_t)(p0 + t) * 2 * Mg + M_L);
-    }
-    cp_async_wait_all();
-    __syncthreads();
-    const C* Lb = Lsm + bx * Q * P + p0;
-#pragma unroll
-    for (int t = 0; t < H; t += 2) {
-        C a0 = zero<C>(), a1 = zero<C>();
-#pragma unroll
-        for (int q = 0; q < Q; ++q) {
-            C l0, l1;
-            if constexpr (sizeof(R) == 4) {
-                const float4 l = *reinterpret_cast<const float4*>(Lb + q * P + t);
-                l0 = make_float2(l.x, l.y); l1 = make_float2(l.z, l.w);
-            } else {
-                l0 = Lb[q * P + t]; l1 = Lb[q * P + t + 1];
-            }
-            rfma(a0, w[q], l0);
-            rfma(a1, w[q], l1);
-        }
-        const int p = p0 + t;
-        if (p > 0) {                                               // C_0 = I (R1)
-            C u = cadd(v[t], a0);
-            u.x -= rr[p].y; u.y += rr[p].x;                        // + i r_p
-            v[t] = cmul(rh[p], u);
-        }
-        C u = cadd(v[t + 1], a1);
-        u.x -= rr[p + 1].y; u.y += rr[p + 1].x;
-        v[t + 1] = cmul(rh[p + 1], u);
-    }
-    // DIF split over the pair: h = 0 forms x[p] + x[p + 32], h = 1 (x[p] - x[p + 32]) w_64^p
-#pragma unroll
-    for (int t = 0; t < H; ++t) {
-        const C o = shfl_xor_c(v[t], 1);                           // partner's value at the same t
-        v[t] = h == 0 ? cadd(v[t], o) : cmul(csub(o, v[t]), tw[t]);
-    }
-    {   // 32-point DFT in registers: 32 = 2 x 16 (even / odd t)
-        C e[16], o[16];
-#pragma unroll
-        for (int t = 0; t < 16; ++t) { e[t] = v[2 * t]; o[t] = v[2 * t + 1]; }
-        dft16(e); dft16(o);
-#pragma unroll
-        for (int k = 0; k < 16; ++k) {
-            const C ow = cmul(o[k], tw[32 + k]);
-            v[k] = cadd(e[k], ow);
-            v[k + 16] = csub(e[k], ow);
-        }
-    }
-    C* dst = W + ((size_t)b << lML) + m;
-#pragma unroll
-    for (int k = 0; k < H; ++k) dst[(size_t)(2 * k + h) * Mg] = v[k];
-}
-
 }  // namespace fmmfft
