@@ -215,6 +215,7 @@ struct fmmfft_plan_s {
     bool inverse = false;            // FMMFFT_FLAG_INVERSE: x = F_N^{-1} y
     bool pp_old = false;
     bool fs_narrow = false;
+    bool pmaj = false;               // M^L / L^L p-major [p][b][q] between k_s2m, k_tree_pc and post_pfft
     int s2t_tpc = 0;                 // FMMFFT_S2T_TPC: tiles per k_s2t_tc CTA (0 = one wave)          // FMMFFT_FS_NARROW=1: 11-bit (c64) / 10-bit (c128) four-step passes on 4-column CTAs             // FMMFFT_PP=tile: the shared-memory-tile k_post_pfft for every P
     bool direct = false;             // FMMFFT_FLAG_DIRECT: plain four-step FFT of length N, no FMM
     bool lvl_off = false;            // FMMFFT_DOWN=tree: every down level in k_tree_down (no k_m2l_lvl)
@@ -677,7 +678,7 @@ struct Exec {
                 if constexpr (!(sizeof(R) == 8 && PCv > 16))
                     dispatch<4, 5, 6, 7>(ilog2(p->M_L), [&](auto lml) {
                         launch_pdl(k_s2m<R, PCv, decltype(lml)::value>, grid, PCv * (Qp / 4) * nbx, smem, s, S, interior(rb.Mpad[p->L]),
-                                   (const R*)p->s2mT, p->P, p->Q, (C*)rb.Sp, (C*)rb.Tn, p->nb, nbx);
+                                   (const R*)p->s2mT, p->P, p->Q, (C*)rb.Sp, (C*)rb.Tn, p->nb, nbx, (int)p->pmaj);
                     });
             });
             LAUNCH_CHECK();
@@ -806,6 +807,7 @@ struct Exec {
             a.L = p->L;
             a.B = p->B;
             a.dbg = (p->flags & FMMFFT_FLAG_DEBUG) ? 1 : 0;
+            a.pmaj = p->pmaj ? 1 : 0;
             const int tabB = ((1 << p->B) - 3) * p->Q * p->Q;
             // complex64 with Q = 16 or 8 and <= 8 boxes per thread group: register-blocked kernel
             if constexpr (sizeof(R) == 4) {
@@ -1117,7 +1119,7 @@ struct Exec {
                         dispatch<8, 16, 24>(p->Q, [&](auto qv) {
                             launch_pdl(k_post_pfft_r<R, LP, decltype(qv)::value>, (unsigned)(p->nb / nbx), nbx * p->M_L, smem, s,
                                        (const C*)rb.Tn, (const C*)rb.Lloc[p->L], (const C*)rb.r, (const C*)p->rho,
-                                       (const R*)p->s2m, (C*)rb.W, ilog2(p->M_L), (int)p->Mg);
+                                       (const R*)p->s2m, (C*)rb.W, ilog2(p->M_L), (int)p->Mg, (int)p->pmaj);
                         });
                     });
                     if (!ok) return fail(FMMFFT_UNSUPPORTED, "k_post_pfft_r: P=%d", p->P);
@@ -1133,8 +1135,8 @@ struct Exec {
         if (p->pp_ms) MS = std::min(p->M_L, p->pp_ms);
         const int threads = std::min(sizeof(R) == 4 ? 1024 : 512, std::max(32, MS * p->P / 8));
         size_t smem = (size_t)MS * (p->P + 1) * sizeof(C) + (size_t)p->P * sizeof(C) + (size_t)p->Q * MS * sizeof(R);
-        const int stage_L = smem + (size_t)p->Q * p->P * sizeof(C) <= 160 * 1024;   // stage L^L of the box
-        if (stage_L) smem += (size_t)p->Q * p->P * sizeof(C);
+        const int stage_L = smem + (size_t)(p->Q + 1) * p->P * sizeof(C) <= 160 * 1024;   // stage L^L of the box
+        if (stage_L) smem += (size_t)(p->Q + 1) * p->P * sizeof(C);
         const int blocks = p->nb * (p->M_L / MS);
         for (RankBufs& rb : p->ranks) {
             const int qt = (p->Q == 8 || p->Q == 16 || p->Q == 24) ? p->Q : 0;
@@ -1143,7 +1145,7 @@ struct Exec {
                 dispatch<0, 8, 16, 24>(qt, [&](auto qv) {
                     launch_pdl(k_post_pfft<R, LP, decltype(qv)::value>, blocks, threads, smem, s, (const C*)rb.Tn,
                                (const C*)rb.Lloc[p->L], (const C*)rb.r, (const C*)p->rho, (const R*)p->s2m, (C*)rb.W,
-                               ilog2(p->M_L), p->Q, ilog2(MS), (int)p->Mg, stage_L);
+                               ilog2(p->M_L), p->Q, ilog2(MS), (int)p->Mg, stage_L, (int)p->pmaj);
                 });
             });
             LAUNCH_CHECK();
@@ -1617,6 +1619,10 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
     // tiles per rank; FMMFFT_S2T=simt selects the FFMA2 kernel (k_near_up) instead
     p->s2t_tc = precision == FMMFFT_C64 && M_L == 64 && (p->nb % S2TC_BOXES) == 0;
     if (const char* e = getenv("FMMFFT_S2T")) p->s2t_tc = p->s2t_tc && e[0] == 't';
+    // the cluster far field gathers M^L and scatters L^L one FMM (one p) at a time: keep both
+    // p-major so those are contiguous runs (debug plans keep [b][q][p] for the stage buffers)
+    p->pmaj = p->tree_p && p->tree_cl > 1 && L > B && !(flags & FMMFFT_FLAG_DEBUG);
+    if (const char* e = getenv("FMMFFT_PMAJ")) p->pmaj = p->pmaj && e[0] != '0';
     if (const char* e = getenv("FMMFFT_DOWN")) p->lvl_off = e[0] == 't';
     if (const char* e = getenv("FMMFFT_PP")) p->pp_old = e[0] == 't';
     if (const char* e = getenv("FMMFFT_S2T_TPC")) p->s2t_tpc = std::max(0, atoi(e));

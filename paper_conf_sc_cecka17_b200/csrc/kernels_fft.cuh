@@ -141,7 +141,7 @@ template <typename R, int LP, int QT>
 __global__ void __launch_bounds__(sizeof(R) == 4 ? 1024 : 512)
 k_post_pfft(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2<R>* __restrict__ r,
             const C2<R>* __restrict__ rho, const R* __restrict__ s2m, C2<R>* __restrict__ W,
-            int lML, int Qrt, int lMS, int Mg, int stage_L) {
+            int lML, int Qrt, int lMS, int Mg, int stage_L, int pmaj) {
     pdl_trigger();
     using C = C2<R>;
     constexpr int P = 1 << LP, LD = P + 1;
@@ -151,8 +151,8 @@ k_post_pfft(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2
     const int MS = 1 << lMS, M_L = 1 << lML;
     C* tile = reinterpret_cast<C*>(smem_raw);                    // [MS][P + 1]
     C* tw = tile + MS * LD;                                       // [P]
-    C* Lsm = tw + P;                                              // [Q][P]   L^L of box b (if staged)
-    R* s2m_sm = reinterpret_cast<R*>(Lsm + (stage_L ? Q * P : 0)); // [Q][MS]  (16-byte aligned: MS % 8 == 0)
+    C* Lsm = tw + P;                                              // [Q][P] (pmaj: [P][Q + 1]) L^L of box b (if staged)
+    R* s2m_sm = reinterpret_cast<R*>(Lsm + (stage_L ? (Q + 1) * P : 0)); // [Q][MS]  (16-byte aligned: MS % 8 == 0)
     const int tid = threadIdx.x, nthr = blockDim.x;
     const int lnsub = lML - lMS;
     const int b = blockIdx.x >> lnsub, m0 = (blockIdx.x & ((1 << lnsub) - 1)) << lMS;
@@ -176,7 +176,13 @@ k_post_pfft(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2
             cp_async_elem(&tile[m * LD + pp].x, src + (size_t)pp * 2 * Mg + m);
             cp_async_elem(&tile[m * LD + pp].y, src + (size_t)pp * 2 * Mg + M_L + m);
         }
-        if (stage_L) {
+        if (stage_L && pmaj) {                                    // [p][b][q] -> Lsm[p][Q + 1] (padded rows)
+            const int nbt = Mg >> lML;
+            for (int idx = tid; idx < Q * P; idx += nthr) {
+                const int pp = idx / Q, q = idx - pp * Q;
+                cp_async_elem(Lsm + pp * (Q + 1) + q, LL + ((size_t)pp * nbt + b) * Q + q);
+            }
+        } else if (stage_L) {
             const C* Lb = LL + (size_t)b * Q * P;
             constexpr int V = 16 / sizeof(C);
             for (int idx = tid; idx < Q * P / V; idx += nthr) cp_async<16>(Lsm + idx * V, Lb + idx * V);
@@ -197,7 +203,8 @@ k_post_pfft(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2
         const R* a = s2m_sm + g * MG;
 #pragma unroll 4
         for (int q = 0; q < Q; ++q) {
-            const C l = stage_L ? Lsm[q * P + p] : ldg_c(Lb + q * P + p);
+            const C l = stage_L ? (pmaj ? Lsm[p * (Q + 1) + q] : Lsm[q * P + p])
+                                : (pmaj ? ldg_c(LL + ((size_t)p * (Mg >> lML) + b) * Q + q) : ldg_c(Lb + q * P + p));
             R av[MG];
             if constexpr (sizeof(R) == 4) {
                 const float4 a0 = *reinterpret_cast<const float4*>(a + q * MS), a1 = *reinterpret_cast<const float4*>(a + q * MS + 4);
@@ -742,7 +749,7 @@ k_conj_scale(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, long long n,
 template <typename R, int LP, int QT>
 __global__ void __launch_bounds__(256)
 k_post_pfft_r(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2<R>* __restrict__ r,
-              const C2<R>* __restrict__ rho, const R* __restrict__ s2m, C2<R>* __restrict__ W, int lML, int Mg) {
+              const C2<R>* __restrict__ rho, const R* __restrict__ s2m, C2<R>* __restrict__ W, int lML, int Mg, int pmaj) {
     pdl_trigger();
     using C = C2<R>;
     constexpr int P = 1 << LP, Q = QT;
@@ -762,8 +769,17 @@ k_post_pfft_r(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const 
     pdl_wait();                                                   // T_near / L^L / r from the FMM stages
     {
         constexpr int V = 16 / sizeof(C);
-        const C* src = LL + (size_t)blockIdx.x * nbx * Q * P;
-        for (int idx = tid; idx < nbx * Q * P / V; idx += blockDim.x) cp_async<16>(Lsm + idx * V, src + idx * V);
+        if (pmaj) {                                               // [p][b][q] -> Lsm[bx][p][q]
+            const int nbt = Mg >> lML;
+            for (int idx = tid; idx < nbx * P * Q / V; idx += blockDim.x) {
+                const int e = idx * V, row = e / Q, q = e - row * Q;  // row = bx P + p
+                const int bxx = row / P, pp = row - bxx * P;
+                cp_async<16>(Lsm + e, LL + ((size_t)pp * nbt + (size_t)blockIdx.x * nbx + bxx) * Q + q);
+            }
+        } else {
+            const C* src = LL + (size_t)blockIdx.x * nbx * Q * P;
+            for (int idx = tid; idx < nbx * Q * P / V; idx += blockDim.x) cp_async<16>(Lsm + idx * V, src + idx * V);
+        }
         if (tid < P) { rr[tid] = ldg_c(r + tid); rh[tid] = ldg_c(rho + tid); }
     }
     C v[P];
@@ -782,7 +798,9 @@ k_post_pfft_r(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const 
 #pragma unroll
         for (int q = 0; q < Q; ++q) {
             C l0, l1;
-            if constexpr (sizeof(R) == 4) {
+            if (pmaj) {                                            // broadcast loads, [p][q]
+                l0 = Lb[p * Q + q]; l1 = Lb[(p + 1) * Q + q];
+            } else if constexpr (sizeof(R) == 4) {
                 const float4 l = *reinterpret_cast<const float4*>(Lb + q * P + p);
                 l0 = make_float2(l.x, l.y); l1 = make_float2(l.z, l.w);
             } else {
