@@ -1790,7 +1790,8 @@ fmmfft_status_t fmmfft_get_info(fmmfft_plan_t p, fmmfft_info_t* info) {
     info->n_stages = ST_COUNT + 1; info->workspace_bytes = p->ws_bytes; info->kernels_per_execute = p->kernels;
     info->variant = (p->tree_p ? FMMFFT_VARIANT_TREE_FUSED : 0u) | (p->s2t_tc ? FMMFFT_VARIANT_S2T_TC : 0u) |
                     ((p->row_fft1 || p->row_cl) ? FMMFFT_VARIANT_ROW_FFT1 : 0u) | (p->fs_lr ? FMMFFT_VARIANT_FOURSTEP : 0u) |
-                    (p->row_cl ? FMMFFT_VARIANT_ROW_CL : 0u) | (!p->tree_p && !p->lvl_off ? FMMFFT_VARIANT_DOWN_LVL : 0u);
+                    (p->row_cl ? FMMFFT_VARIANT_ROW_CL : 0u) | (!p->tree_p && !p->lvl_off ? FMMFFT_VARIANT_DOWN_LVL : 0u) |
+                    (p->pmaj ? FMMFFT_VARIANT_PMAJ : 0u);
     return FMMFFT_SUCCESS;
 }
 

@@ -250,7 +250,11 @@ def test_alternative_paths(F, monkeypatch, env, N, P, B, Q, G):
         Tn = t_near(plan, P, L, 64)
         assert rel(Tn, st["T_near"]) < TOL_STAGE[prec]
         assert np.array_equal(Tn[:, :, 0], x.reshape(2 ** L, 64, P)[:, :, 0])
-        LL = plan.debug_buffer("L", L).cpu().numpy().reshape(2 ** L, Q, P)
+        LL = plan.debug_buffer("L", L).cpu().numpy()
+        if plan.info["variant"] & 64:            # FMMFFT_VARIANT_PMAJ: leaf L^L stored [p][b][q]
+            LL = LL.reshape(P, 2 ** L, Q).transpose(1, 2, 0)
+        else:
+            LL = LL.reshape(2 ** L, Q, P)
         assert rel(LL[:, :, 1:], st["L"][L]) < TOL_STAGE[prec]
 
 
