@@ -78,7 +78,14 @@ template <int N> __device__ __forceinline__ void cp_async_wait_group() {
 // Programmatic dependent launch: let the next kernel in the stream start scheduling its CTAs
 // (call early), and wait until the previous kernel's results are complete and visible (call
 // before the first read of them and before any global write).
+// The explicit early trigger is compiled out: dependents then launch when every CTA of the
+// predecessor has exited (the implicit trigger), which still hides the launch gap but never parks
+// dependent CTAs on SMs the predecessor's later waves (or the side stream) need.
+#ifdef FMMFFT_EARLY_PDL_TRIGGER
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;\n" ::: "memory"); }
+#else
+__device__ __forceinline__ void pdl_trigger() {}
+#endif
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;\n" ::: "memory"); }
 
 }  // namespace fmmfft
