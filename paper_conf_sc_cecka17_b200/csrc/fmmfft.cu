@@ -348,7 +348,6 @@ static fmmfft_status_t build_tables(fmmfft_plan_s* p) {
             return f;
         };
         std::vector<float> tb((size_t)P * S2TC_TAB_FLOATS_PER_P, 0.f);
-        const size_t half = S2TC_B_BYTES / 4;              // floats of one of hi / lo
         for (int pp = 1; pp < P; ++pp) {
             for (int k4 = 0; k4 < 16; ++k4)
                 for (int r = 0; r < S2TC_N; ++r)
@@ -358,9 +357,12 @@ static fmmfft_status_t build_tables(fmmfft_plan_s* p) {
                         const double v = cotpi((double)(pp + (long long)P * d) / (double)N);
                         const float hi = tf32(v);
                         const float lo = tf32(v - (double)hi);
-                        const size_t e = (size_t)pp * S2TC_TAB_FLOATS_PER_P + ((size_t)k4 * (S2TC_N / 8) + r / 8) * 32 + (r % 8) * 4 + kk;
-                        tb[e] = hi;
-                        tb[e + half] = lo;
+                        // rows (seg, hi/lo, i): [Bhi_seg; Blo_seg] contiguous along N
+                        for (int hl = 0; hl < 2; ++hl) {
+                            const int row = seg * 128 + hl * 64 + i;
+                            const size_t e = (size_t)pp * S2TC_TAB_FLOATS_PER_P + ((size_t)k4 * (2 * S2TC_N / 8) + row / 8) * 32 + (row % 8) * 4 + kk;
+                            tb[e] = hl ? lo : hi;
+                        }
                     }
         }
         fmmfft_status_t st2 = dalloc(p, &p->toep, tb.size() * sizeof(float));

@@ -24,7 +24,8 @@
 //              committing each chunk's MMAs to the slot's mbarrier;
 //   warps 4-7  (TMEM lane quarters 0-3) the epilogue: tcgen05.ld of T (re and im accumulators),
 //              coalesced stores through a 32 x 32 shared-memory transpose per warp.
-// Two TMEM accumulator pairs (2 x 128 columns): the epilogue of tile t overlaps the MMAs of t+1.
+// Two TMEM accumulator sets (2 x 256 columns: per component Ahi[Bhi|Blo] in 128 columns, Alo Bhi
+// added to the first 64): the epilogue of tile t overlaps the MMAs of t+1.
 // Output T_near is p-major and planar per box: [p][b][re/im][m] (what k_post_pfft reads).
 // p = 0 (the identity, R1) is written by k_s2m.
 #pragma once
@@ -47,7 +48,12 @@ constexpr int S2TC_A_SLOT = 4 * S2TC_A_PART;              // [re/im][hi/lo] part
 constexpr int S2TC_N = 192;                               // operator rows (segment, i)
 constexpr int S2TC_B_K4 = (S2TC_N / 8) * 128;             // bytes per k4 column of B (24 core matrices)
 constexpr int S2TC_B_BYTES = 16 * S2TC_B_K4;              // one of hi / lo (K = 64)
-constexpr int S2TC_TAB_FLOATS_PER_P = 2 * S2TC_B_BYTES / 4;   // [hi,lo][k4 16][r8 24][8][4]
+constexpr int S2TC_TAB_FLOATS_PER_P = 2 * S2TC_B_BYTES / 4;   // [k4 16][r8 48][8][4], rows (s, hi/lo, i)
+// B rows per k4 column: for each shift s the 64 hi rows then the 64 lo rows, so [Bhi_s; Blo_s] is
+// ONE N = 128 operand: Ahi x [Bhi_s | Blo_s] is one MMA into 128 TMEM columns (the two products
+// summed in the epilogue) and Alo x Bhi_s (N = 64, the same descriptor) accumulates into the first
+// 64 — 2 MMAs per (shift, component, K step) instead of 3, and A_hi is read once.
+constexpr int S2TC_B_K4N = (2 * S2TC_N / 8) * 128;         // bytes per k4 column (48 core matrices)
 constexpr int S2TC_THREADS = 288;
 
 struct S2tcSmem {                                         // byte offsets
@@ -92,7 +98,7 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
         for (int k = 0; k < 12; ++k) tc::mbar_init(&bar[k], (k == 4 || k == 5 || k >= 10) ? 128u : 1u);
         tc::fence_barrier_init();
     }
-    if (warp == 0) tc::tmem_alloc<256>(tmem_slot);
+    if (warp == 0) tc::tmem_alloc<512>(tmem_slot);
     tc::tc_fence_before();
     __syncthreads();
     tc::tc_fence_after();
@@ -169,12 +175,10 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
         if (lane == 0) {
             const float* tp = toep + (size_t)p * S2TC_TAB_FLOATS_PER_P;
             for (int kc = 0; kc < S2TC_NKC; ++kc) {              // B chunk kc: k4 in [4 kc, 4 kc + 4), hi and lo
-                tc::mbar_expect_tx(&bfull[kc], 2 * 4 * S2TC_B_K4);
-                tc::bulk_g2s(Bsm + kc * 4 * S2TC_B_K4, tp + kc * S2TC_B_K4, 4 * S2TC_B_K4, &bfull[kc]);
-                tc::bulk_g2s(Bsm + S2TC_B_BYTES + kc * 4 * S2TC_B_K4, tp + S2TC_B_BYTES / 4 + kc * S2TC_B_K4,
-                             4 * S2TC_B_K4, &bfull[kc]);
+                tc::mbar_expect_tx(&bfull[kc], 4 * S2TC_B_K4N);
+                tc::bulk_g2s(Bsm + kc * 4 * S2TC_B_K4N, tp + kc * S2TC_B_K4N, 4 * S2TC_B_K4N, &bfull[kc]);
             }
-            constexpr uint32_t IDESC = tc::idesc_tf32(128, 64);
+            constexpr uint32_t IDESC128 = tc::idesc_tf32(128, 128), IDESC64 = tc::idesc_tf32(128, 64);
             for (int it = 0; it < nit; ++it) {
                 const int buf = it & 1;
                 if (it >= 2) tc::mbar_wait(&aempty[buf], ((it >> 1) + 1) & 1);   // epilogue of tile it-2 done
@@ -186,21 +190,19 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
                     const unsigned char* As = Asm + slot * S2TC_A_SLOT;
 #pragma unroll
                     for (int st = 0; st < S2TC_KC / 8; ++st) {
-                        const unsigned char* bk = Bsm + (4 * kc + 2 * st) * S2TC_B_K4;
+                        const unsigned char* bk = Bsm + (4 * kc + 2 * st) * S2TC_B_K4N;
 #pragma unroll
                         for (int c = 0; c < 2; ++c) {
-                            const uint32_t d = tmem + (uint32_t)(buf * 128 + c * 64);
+                            const uint32_t d = tmem + (uint32_t)(buf * 256 + c * 128);
                             const unsigned char* ahp = As + (2 * c) * S2TC_A_PART + 2 * st * S2TC_LBO_A;
                             const unsigned char* alp = As + (2 * c + 1) * S2TC_A_PART + 2 * st * S2TC_LBO_A;
 #pragma unroll
                             for (int s = 0; s < 3; ++s) {        // rows of boxes b0-1+s ..: 16-byte offset
                                 const uint64_t ah = tc::umma_desc_kmajor(ahp + 16 * s, S2TC_LBO_A, 128);
                                 const uint64_t al = tc::umma_desc_kmajor(alp + 16 * s, S2TC_LBO_A, 128);
-                                const uint64_t bh = tc::umma_desc_kmajor(bk + s * 1024, S2TC_B_K4, 128);
-                                const uint64_t blo = tc::umma_desc_kmajor(bk + S2TC_B_BYTES + s * 1024, S2TC_B_K4, 128);
-                                tc::mma_tf32(d, ah, bh, IDESC, (kc | st | s) ? 1u : 0u);
-                                tc::mma_tf32(d, ah, blo, IDESC, 1u);
-                                tc::mma_tf32(d, al, bh, IDESC, 1u);
+                                const uint64_t b2 = tc::umma_desc_kmajor(bk + s * 2048, S2TC_B_K4N, 128);   // [Bhi_s; Blo_s]
+                                tc::mma_tf32(d, ah, b2, IDESC128, (kc | st | s) ? 1u : 0u);
+                                tc::mma_tf32(d, al, b2, IDESC64, 1u);                                      // Alo Bhi_s
                             }
                         }
                     }
@@ -227,7 +229,13 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
             for (int ch = 0; ch < 4; ++ch) {                     // (component, i half)
                 const int c = ch >> 1, h = ch & 1;
                 float v[32];
-                tc::tmem_ld32(tmem + ((uint32_t)(32 * q) << 16) + (uint32_t)(buf * 128 + c * 64 + 32 * h), v);
+                tc::tmem_ld32(tmem + ((uint32_t)(32 * q) << 16) + (uint32_t)(buf * 256 + c * 128 + 32 * h), v);
+                {   // + the Ahi Blo half (columns 64..127 of the component)
+                    float v2[32];
+                    tc::tmem_ld32(tmem + ((uint32_t)(32 * q) << 16) + (uint32_t)(buf * 256 + c * 128 + 64 + 32 * h), v2);
+#pragma unroll
+                    for (int k = 0; k < 32; ++k) v[k] += v2[k];
+                }
                 if (ch == 3) {                                   // accumulators free for tile it + 2
                     tc::tc_fence_before();
                     tc::mbar_arrive(&aempty[buf]);
@@ -245,7 +253,7 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
     tc::tc_fence_before();
     __syncthreads();
     STAMP(40);
-    if (warp == 0) tc::tmem_dealloc<256>(tmem);
+    if (warp == 0) tc::tmem_dealloc<512>(tmem);
 }
 
 }  // namespace fmmfft
