@@ -215,10 +215,10 @@ struct fmmfft_plan_s {
     int fs_lc1 = 0, fs_lc2 = 0, fs_lr = 0;   // four-step large-M FFT: column pass bits (2nd: 0 = none), row pass bits
     int s2m_nbx = 0, s2m_pc = 0, pp_ms = 0;  // tuning knobs (FMMFFT_S2M_NBX, FMMFFT_S2M_PC, FMMFFT_PP_MS); 0 = default
     bool inverse = false;            // FMMFFT_FLAG_INVERSE: x = F_N^{-1} y
-    bool pp_old = false;
-    bool fs_narrow = false;
+    bool pp_old = false;             // FMMFFT_PP=tile: the shared-memory-tile k_post_pfft for every P
+    bool fs_narrow = false;          // FMMFFT_FS_NARROW=1: 11-bit (c64) / 10-bit (c128) four-step passes on 4-column CTAs
     bool pmaj = false;               // M^L / L^L p-major [p][b][q] between k_s2m, k_tree_pc and post_pfft
-    int s2t_tpc = 0;                 // FMMFFT_S2T_TPC: tiles per k_s2t_tc CTA (0 = one wave)          // FMMFFT_FS_NARROW=1: 11-bit (c64) / 10-bit (c128) four-step passes on 4-column CTAs             // FMMFFT_PP=tile: the shared-memory-tile k_post_pfft for every P
+    int s2t_tpc = 0;                 // FMMFFT_S2T_TPC: tiles per k_s2t_tc CTA (0 = one wave)
     bool direct = false;             // FMMFFT_FLAG_DIRECT: plain four-step FFT of length N, no FMM
     bool lvl_off = false;            // FMMFFT_DOWN=tree: every down level in k_tree_down (no k_m2l_lvl)
     bool s2t_tc = false;             // S2T on tcgen05 (k_s2t_tc): complex64, M_L = 64, nb % 128 == 0
@@ -524,7 +524,7 @@ static fmmfft_status_t init_kernel_attrs() {
             set((const void*)k_tree_pc<8, 512, 2>);
             set((const void*)k_tree_pc<8, 256, 4>);
         }
-        if constexpr (sizeof(R) == 4) set((const void*)k_s2t_tc);
+        if constexpr (sizeof(R) == 4) { set((const void*)k_s2t_tc<1>); set((const void*)k_s2t_tc<2>); }
         set((const void*)k_base_sg<R, 4, sizeof(R) == 4 ? 8 : 4, 4>);
         for (int lp = 1; lp <= 5; ++lp)
             dispatch<1, 2, 3, 4, 5>(lp, [&](auto v) {
@@ -704,8 +704,14 @@ struct Exec {
                 if (p->s2t_tpc) tpc = std::min(ntile, p->s2t_tpc);
                 for (RankBufs& rb : p->ranks) {
                     const dim3 grid((unsigned)((ntile + tpc - 1) / tpc), (unsigned)(p->P - 1));
-                    launch_pdl(k_s2t_tc, grid, S2TC_THREADS, s2tc_smem_bytes(), p->side, (const C*)rb.Sp, (const C*)rb.haloL,
-                               (const C*)rb.haloR, (float*)rb.Tn, (const float*)p->toep, p->P, p->nb, p->G, tpc);
+                    // several tiles per CTA: A chunks prefetched two ahead; one tile: one ahead (the
+                    // first chunk's loads alone, so the first MMAs start sooner)
+                    if (tpc > 1)
+                        launch_pdl(k_s2t_tc<2>, grid, S2TC_THREADS, s2tc_smem_bytes(), p->side, (const C*)rb.Sp, (const C*)rb.haloL,
+                                   (const C*)rb.haloR, (float*)rb.Tn, (const float*)p->toep, p->P, p->nb, p->G, tpc);
+                    else
+                        launch_pdl(k_s2t_tc<1>, grid, S2TC_THREADS, s2tc_smem_bytes(), p->side, (const C*)rb.Sp, (const C*)rb.haloL,
+                                   (const C*)rb.haloR, (float*)rb.Tn, (const float*)p->toep, p->P, p->nb, p->G, tpc);
                     LAUNCH_CHECK();
                 }
                 if ((st = mark_on(p->ev_s2t[1], p->side))) return st;

@@ -66,6 +66,7 @@ struct S2tcSmem {                                         // byte offsets
 };
 __host__ __device__ constexpr size_t s2tc_smem_bytes() { return (size_t)S2tcSmem::TOTAL; }
 
+template <int PF>                                          // A-chunk prefetch distance (1 or 2)
 __global__ void __launch_bounds__(S2TC_THREADS, 1)
 k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const float2* __restrict__ haloR,
          float* __restrict__ Tn, const float* __restrict__ toep, int P, int nb, int G, int tiles_per_cta) {
@@ -109,8 +110,8 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
         // ------------------------------------------------------------ A builders (128 threads)
         // item j: row r = idx >> 2 (box b0 - 1 + r), k4 = idx & 3, idx = tid + 128 j < 4 x 130
         constexpr int NJ = (4 * S2TC_ROWS + 127) / 128;          // 5
-        float4 sv[NJ][2];
-        auto load_chunk = [&](int t, int kc) {
+        float4 sv[2][NJ][2];                                     // two chunks in flight (prefetch distance 2)
+        auto load_chunk = [&](float4 (&svb)[NJ][2], int t, int kc) {
 #pragma unroll
             for (int j = 0; j < NJ; ++j) {
                 const int idx = tid + 128 * j;
@@ -120,23 +121,25 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
                     const int m = S2TC_KC * kc + 4 * k4;
                     if (g >= 0 && g < nb) {
                         const float4* src = reinterpret_cast<const float4*>(spp + (size_t)g * 64 + m);
-                        sv[j][0] = __ldg(src);
-                        sv[j][1] = __ldg(src + 1);
+                        svb[j][0] = __ldg(src);
+                        svb[j][1] = __ldg(src + 1);
                     } else if (G == 1) {                         // periodic wrap (R8)
                         const float4* src = reinterpret_cast<const float4*>(spp + (size_t)((g + nb) % nb) * 64 + m);
-                        sv[j][0] = __ldg(src);
-                        sv[j][1] = __ldg(src + 1);
+                        svb[j][0] = __ldg(src);
+                        svb[j][1] = __ldg(src + 1);
                     } else {                                     // neighbour rank's box ([m][P] layout)
                         const float2* h = (g < 0 ? haloL : haloR) + (size_t)m * P + p;
                         const float2 a = __ldg(h), b = __ldg(h + P), c = __ldg(h + 2 * P), d = __ldg(h + 3 * P);
-                        sv[j][0] = make_float4(a.x, a.y, b.x, b.y);
-                        sv[j][1] = make_float4(c.x, c.y, d.x, d.y);
+                        svb[j][0] = make_float4(a.x, a.y, b.x, b.y);
+                        svb[j][1] = make_float4(c.x, c.y, d.x, d.y);
                     }
                 }
             }
         };
-        load_chunk(t0, 0);
+        load_chunk(sv[0], t0, 0);
+        if (PF == 2) load_chunk(sv[1], t0, 1);
         for (int it = 0; it < nit; ++it) {
+#pragma unroll
             for (int kc = 0; kc < S2TC_NKC; ++kc) {
                 const int gi = it * S2TC_NKC + kc, slot = gi & 1, use = gi >> 1;
                 if (use > 0) tc::mbar_wait(&cempty[slot], (use - 1) & 1);   // MMAs done with this slot
@@ -146,7 +149,7 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
                     const int idx = tid + 128 * j;
                     if (idx < 4 * S2TC_ROWS) {
                         const int r = idx >> 2, k4 = idx & 3;
-                        const float4 u0 = sv[j][0], u1 = sv[j][1];   // (re, im) of 4 consecutive m
+                        const float4 u0 = sv[kc & 1][j][0], u1 = sv[kc & 1][j][1];   // (re, im) of 4 consecutive m
                         const float re[4] = {u0.x, u0.z, u1.x, u1.z}, im[4] = {u0.y, u0.w, u1.y, u1.w};
                         float4 rh, rl, ihv, il;
                         float* prh = &rh.x; float* prl = &rl.x; float* pih = &ihv.x; float* pil = &il.x;
@@ -165,9 +168,9 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
                 tc::fence_proxy_async();
                 tc::mbar_arrive(&cfull[slot]);
                 if (it < 2) STAMP(41 + 4 * it + kc);
-                // prefetch the next chunk (next tile's first chunk after the last one)
-                if (kc + 1 < S2TC_NKC) load_chunk(t0 + it, kc + 1);
-                else if (it + 1 < nit) load_chunk(t0 + it + 1, 0);
+                // prefetch chunk kc + PF (into the buffer just consumed when PF = 2; S2TC_NKC is even)
+                if (kc + PF < S2TC_NKC) load_chunk(sv[(kc + PF) & 1], t0 + it, kc + PF);
+                else if (it + 1 < nit) load_chunk(sv[(kc + PF) & 1], t0 + it + 1, kc + PF - S2TC_NKC);
             }
         }
     } else if (warp == 8) {

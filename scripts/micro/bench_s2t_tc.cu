@@ -19,14 +19,15 @@ int main(int argc, char** argv) {
     cudaMalloc(&Sp, n * 8); cudaMalloc(&Tn, n * 8);
     cudaMalloc(&toep, (size_t)P * S2TC_TAB_FLOATS_PER_P * 4); cudaMalloc(&kf, (size_t)P * 1024);
     cudaMemset(Sp, 0, n * 8); cudaMemset(toep, 0, (size_t)P * S2TC_TAB_FLOATS_PER_P * 4); cudaMemset(kf, 0, (size_t)P * 1024);
-    cudaFuncSetAttribute(k_s2t_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)s2tc_smem_bytes());
+    cudaFuncSetAttribute(k_s2t_tc<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)s2tc_smem_bytes());
+    cudaFuncSetAttribute(k_s2t_tc<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)s2tc_smem_bytes());
     int ntile = nb / S2TC_BOXES;
     dim3 grid((ntile + tpc - 1) / tpc, P - 1);
     cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
-    for (int i = 0; i < 5; ++i) k_s2t_tc<<<grid, S2TC_THREADS, s2tc_smem_bytes()>>>(Sp, Sp, Sp, (float*)Tn, toep, P, nb, 1, tpc);
+    for (int i = 0; i < 5; ++i) (tpc > 1 ? k_s2t_tc<2> : k_s2t_tc<1>)<<<grid, S2TC_THREADS, s2tc_smem_bytes()>>>(Sp, Sp, Sp, (float*)Tn, toep, P, nb, 1, tpc);
     cudaEventRecord(a);
     const int R = 50;
-    for (int i = 0; i < R; ++i) k_s2t_tc<<<grid, S2TC_THREADS, s2tc_smem_bytes()>>>(Sp, Sp, Sp, (float*)Tn, toep, P, nb, 1, tpc);
+    for (int i = 0; i < R; ++i) (tpc > 1 ? k_s2t_tc<2> : k_s2t_tc<1>)<<<grid, S2TC_THREADS, s2tc_smem_bytes()>>>(Sp, Sp, Sp, (float*)Tn, toep, P, nb, 1, tpc);
     cudaEventRecord(b); cudaEventSynchronize(b);
     float ms; cudaEventElapsedTime(&ms, a, b);
     printf("nb=%d P=%d tpc=%d grid=%dx%d: %.2f us/launch  err=%s\n", nb, P, tpc, grid.x, grid.y, ms * 1e3 / R,
