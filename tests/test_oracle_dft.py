@@ -143,3 +143,31 @@ def test_inverse_roundtrip_and_radix2(N):
     assert O.rel_l2(O.fft_radix2(y, inverse=True), x) < 1e-13
     assert O.rel_l2(O.fft_radix2(x, inverse=True), O.dft_direct(x, inverse=True)) < 1e-13
     assert O.rel_l2(O.fft_radix2(x, inverse=True), np.fft.ifft(x)) < 1e-13
+
+
+# ---- real-input transform (SURVEY §8(f) NEXT-1, C = 1)
+
+@pytest.mark.parametrize("N", [2, 16, 1024, 24])
+def test_rdft_vs_numpy_and_hermitian(N):
+    rng = np.random.default_rng(N)
+    x = rng.standard_normal(N)
+    y = O.rdft(x)
+    assert y.shape == (N // 2 + 1,)
+    # independent library routine
+    assert np.max(np.abs(y - np.fft.rfft(x))) < 1e-12 * max(1, np.sqrt(N))
+    # the full DFT of a real vector is Hermitian: y_{N-k} = conj(y_k); y_0, y_{N/2} real
+    full = O.dft_direct(x.astype(complex))
+    assert np.max(np.abs(full[1:][::-1] - np.conj(full[1:]))) < 1e-10
+    assert abs(y[0].imag) < 1e-12 and abs(y[-1].imag) < 1e-10
+    assert abs(y[0] - x.sum()) < 1e-10
+    assert abs(y[-1] - (x[0::2].sum() - x[1::2].sum())) < 1e-10
+
+
+@pytest.mark.parametrize("N,k0", [(64, 5), (4096, 1000)])
+def test_rdft_cosine(N, k0):
+    # x_j = cos(2 pi k0 j / N) -> y_k0 = N/2, every other k in 0..N/2 zero
+    j = np.arange(N)
+    y = O.rdft(np.cos(2 * np.pi * ((k0 * j) % N) / N))
+    expect = np.zeros(N // 2 + 1, dtype=complex)
+    expect[k0] = N / 2
+    assert np.max(np.abs(y - expect)) < 1e-10 * N
