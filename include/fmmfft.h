@@ -79,6 +79,19 @@ typedef enum {
                                    (two extra elementwise passes, k_conj_scale). Same layouts,
                                    distribution and error bounds as the forward plan. */
 
+#define FMMFFT_FLAG_REAL 32u    /* real-input forward transform (C = 1):
+                                   X_k = sum_j x_j exp(-2 pi i jk/N), k = 0..N/2, for REAL x
+                                   (eq. 1; the other half is conj(X_{N-k})).
+                                   N is the real length (even); in = N reals (float / double by
+                                   precision, 16-byte aligned), out = N/2 + 1 complex values
+                                   (must not overlap in). The N reals are read in place as the
+                                   complex vector z_j = x_{2j} + i x_{2j+1}, transformed by the
+                                   complex plan of length N/2 (P, B, Q, M_L — or DIRECT — apply
+                                   to THAT length), then one elementwise pass (k_r2c_post)
+                                   separates the even / odd halves. G = 1 only, not with
+                                   INVERSE / VIRTUAL (else FMMFFT_UNSUPPORTED). fmmfft_get_info
+                                   reports the real N; M, L, ... describe the complex plan. */
+
 /* ---------------------------------------------------------------- communicator (G > 1)
  * One process per GPU. Rank 0 calls fmmfft_get_unique_id and broadcasts the 128 bytes (e.g.
  * through torch.distributed); every rank then calls fmmfft_comm_init with its rank, the

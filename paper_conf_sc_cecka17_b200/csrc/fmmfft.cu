@@ -176,6 +176,7 @@ struct RankBufs {
     void* haloR = nullptr;   // S box nb  (G > 1)
     void* r = nullptr;       // [P] reductions
     void* cin = nullptr;     // conj(in) (inverse plans)
+    void* rz = nullptr;      // Z = F_{N/2} z (real-input plans, FMMFFT_FLAG_REAL)
     void* din = nullptr;     // execute_host staging
     void* dout = nullptr;
     std::vector<void*> Mpad, Lloc, Mfull, Lfull;   // indexed by level
@@ -215,6 +216,7 @@ struct fmmfft_plan_s {
     int fs_lc1 = 0, fs_lc2 = 0, fs_lr = 0;   // four-step large-M FFT: column pass bits (2nd: 0 = none), row pass bits
     int s2m_nbx = 0, s2m_pc = 0, pp_ms = 0;  // tuning knobs (FMMFFT_S2M_NBX, FMMFFT_S2M_PC, FMMFFT_PP_MS); 0 = default
     bool inverse = false;            // FMMFFT_FLAG_INVERSE: x = F_N^{-1} y
+    bool real = false;               // FMMFFT_FLAG_REAL: N (below) is the complex length H = N_real / 2
     bool pp_old = false;             // FMMFFT_PP=tile: the shared-memory-tile k_post_pfft for every P
     bool fs_narrow = false;          // FMMFFT_FS_NARROW=1: 11-bit (c64) / 10-bit (c128) four-step passes on 4-column CTAs
     bool pmaj = false;               // M^L / L^L p-major [p][b][q] between k_s2m, k_tree_pc and post_pfft
@@ -1318,8 +1320,23 @@ struct Exec {
         return FMMFFT_SUCCESS;
     }
 
+    // real-input plans: X_k, k = 0..H, from Z = F_H z (k_r2c_post)
+    fmmfft_status_t r2c_post(const C* Z, C* X) {
+        const long long H = p->N;
+        const unsigned blocks = (unsigned)std::min<long long>((H / 2 + 256) / 256, 148LL * 8);
+        launch_pdl(k_r2c_post<R>, blocks, 256, 0, s, Z, X, H);
+        LAUNCH_CHECK();
+        return FMMFFT_SUCCESS;
+    }
+
     fmmfft_status_t run() {
         fmmfft_status_t st;
+        if (p->real) {                                  // z_j = x_{2j} + i x_{2j+1}: the input as is
+            C* X = out[0];
+            out[0] = (C*)p->ranks[0].rz;
+            if ((st = run_forward())) return st;
+            return r2c_post(out[0], X);
+        }
         if (p->inverse)                                 // F^{-1} x = conj(F conj(x)) / N
             for (RankBufs& rb : p->ranks) {
                 const int g = p->virt ? rb.g : 0;
@@ -1558,8 +1575,8 @@ static fmmfft_status_t plan_direct(fmmfft_plan_t* plan, long long N, int G, fmmf
     return FMMFFT_SUCCESS;
 }
 
-fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, int B, int Q,
-                               fmmfft_precision_t precision, int M_L, unsigned flags) {
+static fmmfft_status_t plan_complex(fmmfft_plan_t* plan, long long N, int P, int G, int B, int Q,
+                                    fmmfft_precision_t precision, int M_L, unsigned flags) {
     if (!plan) return fail(FMMFFT_INVALID_VALUE, "plan is NULL");
     *plan = nullptr;
     if (precision != FMMFFT_C64 && precision != FMMFFT_C128) return fail(FMMFFT_INVALID_VALUE, "bad precision");
@@ -1747,6 +1764,30 @@ fmmfft_status_t fmmfft_autotune(long long N, int G, fmmfft_precision_t precision
     return FMMFFT_SUCCESS;
 }
 
+// FMMFFT_FLAG_REAL (SURVEY §8(f) NEXT-1, C = 1): N real inputs read as the complex vector
+// z_j = x_{2j} + i x_{2j+1} of length H = N/2, the complex plan of length H (FMM or DIRECT), then
+// k_r2c_post. G = 1 only; no INVERSE / VIRTUAL.
+fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, int B, int Q,
+                               fmmfft_precision_t precision, int M_L, unsigned flags) {
+    if (!(flags & FMMFFT_FLAG_REAL)) return plan_complex(plan, N, P, G, B, Q, precision, M_L, flags);
+    if (!plan) return fail(FMMFFT_INVALID_VALUE, "plan is NULL");
+    *plan = nullptr;
+    if (G != 1) return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_REAL: single GPU only (G = 1)");
+    if (flags & (FMMFFT_FLAG_INVERSE | FMMFFT_FLAG_VIRTUAL))
+        return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_REAL: forward, non-virtual plans only");
+    if (N < 4 || (N & 1)) return fail(FMMFFT_INVALID_VALUE, "FMMFFT_FLAG_REAL: N must be even");
+    fmmfft_status_t st = plan_complex(plan, N / 2, P, G, B, Q, precision, M_L, flags);
+    if (st) return st;
+    fmmfft_plan_s* p = *plan;
+    p->real = true;
+    if ((st = dalloc(p, &p->ranks[0].rz, (size_t)(N / 2) * p->esz))) {
+        destroy_plan(p);
+        *plan = nullptr;
+        return st;
+    }
+    return FMMFFT_SUCCESS;
+}
+
 fmmfft_status_t fmmfft_plan(fmmfft_plan_t* plan, long long N, int P, int G, int B, int Q, fmmfft_precision_t precision) {
     return fmmfft_plan_ex(plan, N, P, G, B, Q, precision, 64, 0u);
 }
@@ -1755,9 +1796,10 @@ fmmfft_status_t fmmfft_execute(fmmfft_plan_t p, const void* in, void* out, void*
     if (!p) return fail(FMMFFT_INVALID_VALUE, "plan is NULL");
     if (!in || !out) return fail(FMMFFT_INVALID_VALUE, "in/out is NULL");
     const size_t bytes = (size_t)(p->virt ? p->N : p->N / p->G) * p->esz;
+    const size_t obytes = bytes + (p->real ? p->esz : 0);   // real plans: N/2 + 1 outputs
     const char* a = (const char*)in;
     const char* b = (const char*)out;
-    if (a < b + bytes && b < a + bytes) return fail(FMMFFT_INVALID_VALUE, "in and out overlap");
+    if (a < b + obytes && b < a + bytes) return fail(FMMFFT_INVALID_VALUE, "in and out overlap");
     if (((uintptr_t)in | (uintptr_t)out) & 15) return fail(FMMFFT_INVALID_VALUE, "in/out must be 16-byte aligned");
     cudaPointerAttributes at;
     if (cudaPointerGetAttributes(&at, in) != cudaSuccess || at.type != cudaMemoryTypeDevice ||
@@ -1772,17 +1814,18 @@ fmmfft_status_t fmmfft_execute(fmmfft_plan_t p, const void* in, void* out, void*
 fmmfft_status_t fmmfft_execute_host(fmmfft_plan_t p, const void* in_host, void* out_host, void* stream) {
     if (!p || !in_host || !out_host) return fail(FMMFFT_INVALID_VALUE, "NULL argument");
     const size_t bytes = (size_t)(p->virt ? p->N : p->N / p->G) * p->esz;
+    const size_t obytes = bytes + (p->real ? p->esz : 0);   // real plans: N/2 + 1 outputs
     RankBufs& rb = p->ranks[0];
     if (!rb.din) {
         fmmfft_status_t st;
         if ((st = dalloc(p, &rb.din, bytes))) return st;
-        if ((st = dalloc(p, &rb.dout, bytes))) return st;
+        if ((st = dalloc(p, &rb.dout, obytes))) return st;
     }
     cudaStream_t s = (cudaStream_t)stream;
     CUDA_TRY(cudaMemcpyAsync(rb.din, in_host, bytes, cudaMemcpyHostToDevice, s));
     fmmfft_status_t st = p->prec == FMMFFT_C64 ? execute_t<float>(p, rb.din, rb.dout, s) : execute_t<double>(p, rb.din, rb.dout, s);
     if (st) return st;
-    CUDA_TRY(cudaMemcpyAsync(out_host, rb.dout, bytes, cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaMemcpyAsync(out_host, rb.dout, obytes, cudaMemcpyDeviceToHost, s));
     return FMMFFT_SUCCESS;
 }
 
@@ -1795,7 +1838,7 @@ fmmfft_status_t fmmfft_destroy(fmmfft_plan_t p) {
 
 fmmfft_status_t fmmfft_get_info(fmmfft_plan_t p, fmmfft_info_t* info) {
     if (!p || !info) return fail(FMMFFT_INVALID_VALUE, "NULL argument");
-    info->N = p->N; info->P = p->P; info->G = p->G; info->B = p->B; info->Q = p->Q; info->M_L = p->M_L;
+    info->N = p->real ? 2 * p->N : p->N; info->P = p->P; info->G = p->G; info->B = p->B; info->Q = p->Q; info->M_L = p->M_L;
     info->L = p->L; info->precision = p->prec; info->M = p->M; info->level_gather = p->lg;
     info->n_stages = ST_COUNT + 1; info->workspace_bytes = p->ws_bytes; info->kernels_per_execute = p->kernels;
     info->variant = (p->tree_p ? FMMFFT_VARIANT_TREE_FUSED : 0u) | (p->s2t_tc ? FMMFFT_VARIANT_S2T_TC : 0u) |

@@ -739,6 +739,41 @@ k_conj_scale(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, long long n,
 }
 
 // ---------------------------------------------------------------------------------------------
+// k_r2c_post (FMMFFT_FLAG_REAL): real x of length N = 2H read as the complex
+// vector z_j = x_{2j} + i x_{2j+1}; Z = F_H z comes from the complex plan. With a = Z_k,
+// b = conj(Z_{H-k}) (Z_H = Z_0): E = (a + b)/2 (the DFT of the even samples), O = -i (a - b)/2
+// (of the odd ones), and eq. (1) split by parity gives X_k = E + w_N^k O and
+// X_{H-k} = conj(E - w_N^k O). Thread k <= H/2 reads Z_k and Z_{H-k} and writes both outputs,
+// so every element is read and written once (coalesced, the second stream descending).
+// ---------------------------------------------------------------------------------------------
+template <typename R>
+__global__ void __launch_bounds__(256)
+k_r2c_post(const C2<R>* __restrict__ Z, C2<R>* __restrict__ X, long long H) {
+    pdl_trigger();
+    pdl_wait();
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    for (long long k = (long long)blockIdx.x * blockDim.x + threadIdx.x; k <= H / 2; k += stride) {
+        const C2<R> a = Z[k];
+        const C2<R> zb = Z[k == 0 ? 0 : H - k];
+        const R Er = R(0.5) * (a.x + zb.x), Ei = R(0.5) * (a.y - zb.y);   // (a + conj(zb)) / 2
+        const R Or = R(0.5) * (a.y + zb.y), Oi = R(-0.5) * (a.x - zb.x);  // -i (a - conj(zb)) / 2
+        R wr, wi;                                                        // w_N^k = exp(-2 pi i k / 2H)
+        if constexpr (sizeof(R) == 4) {
+            float sn, cs;
+            sincospif(-(float)((double)k / (double)H), &sn, &cs);
+            wr = cs; wi = sn;
+        } else {
+            double sn, cs;
+            sincospi(-(double)k / (double)H, &sn, &cs);
+            wr = cs; wi = sn;
+        }
+        const R tr = wr * Or - wi * Oi, ti = wr * Oi + wi * Or;            // w O
+        X[k] = C2<R>{Er + tr, Ei + ti};
+        X[H - k] = C2<R>{Er - tr, -(Ei - ti)};
+    }
+}
+
+// ---------------------------------------------------------------------------------------------
 // k_post_pfft_r: the same L2T + POST + P-point FFT + transposed store for P <= 32 with the whole
 // P-point column of one m in one thread's registers (no shared-memory FFT tile, no barriers in
 // the FFT): thread (box b, m) loads T_near[p][b][.][m] for all p (coalesced over m), adds

@@ -15,7 +15,7 @@ import ctypes
 import torch
 
 from . import _lib
-from ._lib import C64, C128, FLAG_DEBUG, FLAG_DIRECT, FLAG_INVERSE, FLAG_PROFILE, FLAG_VIRTUAL, check, lib
+from ._lib import C64, C128, FLAG_DEBUG, FLAG_DIRECT, FLAG_INVERSE, FLAG_PROFILE, FLAG_REAL, FLAG_VIRTUAL, check, lib
 
 _DT = {"c64": (C64, torch.complex64), "c128": (C128, torch.complex128)}
 
@@ -68,16 +68,20 @@ class _DevView:
 class FmmFFT:
     def __init__(self, N: int, P: int, G: int = 1, B: int = 2, Q: int = 16, precision: str = "c64",
                  M_L: int = 64, virtual: bool = False, profile: bool = False, debug: bool = False,
-                 inverse: bool = False, direct: bool = False):
+                 inverse: bool = False, direct: bool = False, real: bool = False):
         """direct=True: no FMM — the plain four-step FFT of length N on one GPU with the same M-FFT
-        kernels (the in-house Cooley-Tukey comparator; P, B, Q, M_L ignored)."""
+        kernels (the in-house Cooley-Tukey comparator; P, B, Q, M_L ignored).
+        real=True (FMMFFT_FLAG_REAL): N real inputs -> N/2+1 complex outputs; P, B, Q, M_L
+        describe the complex plan of length N/2 (G = 1)."""
         self.N, self.P, self.G, self.B, self.Q, self.M_L = N, P, G, B, Q, M_L
         self.precision = precision
         self.virtual = virtual
         self._prec, self.dtype = _DT[precision]
         flags = (FLAG_VIRTUAL if virtual else 0) | (FLAG_PROFILE if profile else 0) | (FLAG_DEBUG if debug else 0) | \
-                (FLAG_INVERSE if inverse else 0) | (FLAG_DIRECT if direct else 0)
+                (FLAG_INVERSE if inverse else 0) | (FLAG_DIRECT if direct else 0) | (FLAG_REAL if real else 0)
         self.inverse = inverse
+        self.real = real
+        self.in_dtype = (torch.float32 if precision == "c64" else torch.float64) if real else self.dtype
         h = ctypes.c_void_p()
         check(lib.fmmfft_plan_ex(ctypes.byref(h), N, P, G, B, Q, self._prec, M_L, flags))
         self._h = h
@@ -85,10 +89,13 @@ class FmmFFT:
 
     # -- execution
     def __call__(self, x: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
-        if x.dtype != self.dtype or not x.is_cuda or not x.is_contiguous() or x.numel() != self.n_local:
-            raise ValueError(f"expected a contiguous CUDA {self.dtype} tensor of {self.n_local} elements")
+        if x.dtype != self.in_dtype or not x.is_cuda or not x.is_contiguous() or x.numel() != self.n_local:
+            raise ValueError(f"expected a contiguous CUDA {self.in_dtype} tensor of {self.n_local} elements")
+        n_out = self.N // 2 + 1 if self.real else self.n_local
         if out is None:
-            out = torch.empty_like(x)
+            out = torch.empty(n_out, dtype=self.dtype, device=x.device)
+        elif out.dtype != self.dtype or not out.is_contiguous() or out.numel() != n_out:
+            raise ValueError(f"out must be a contiguous {self.dtype} tensor of {n_out} elements")
         check(lib.fmmfft_execute(self._h, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(out.data_ptr()),
                                  _stream_ptr(stream)))
         return out

@@ -58,6 +58,12 @@ def complex_uniform(n0: int, count: int, seed: int = DEFAULT_SEED,
     return out
 
 
+def real_uniform(n0: int, count: int, seed: int = DEFAULT_SEED, dtype=np.float64) -> np.ndarray:
+    """Real inputs x[n0 : n0+count] (FMMFFT_FLAG_REAL), uniform on [-1, 1), as ``dtype``."""
+    n = np.arange(n0, n0 + count, dtype=np.uint64)
+    return uniform_pm1(seed, n).astype(dtype)
+
+
 def shard(N: int, G: int, rank: int, seed: int = DEFAULT_SEED, dtype=np.complex128) -> np.ndarray:
     """Rank ``rank``'s block of the length-N input: x[rank*N/G : (rank+1)*N/G]."""
     assert N % G == 0

@@ -331,3 +331,40 @@ def test_post_pfft_variants(F, monkeypatch, env, P, Q, prec):
     N = 1 << 18
     plan, x, y = run(F, N, P, 2, Q, prec, 64)
     assert rel(y, O.fft_radix2(x)) < (1e-5 if prec == "c64" else 1e-11)
+
+
+# ------------------------------------------------------------------ real input, C = 1 (§8(f) NEXT-1)
+@pytest.mark.parametrize("N,P,B,Q,prec,direct", [
+    (1 << 13, 16, 2, 16, "c128", False),   # complex plan = cfg1 (N/2 = 2^12)
+    (1 << 13, 16, 2, 16, "c64", False),
+    (1 << 21, 64, 2, 16, "c64", False),    # complex plan = cfg2
+    (1 << 21, 64, 2, 16, "c128", False),
+    (1 << 16, 1, 2, 16, "c64", True),      # four-step (DIRECT) complex plan
+    (1 << 16, 1, 2, 16, "c128", True),
+])
+def test_real_input_vs_oracle(F, N, P, B, Q, prec, direct):
+    rdt = np.float32 if prec == "c64" else np.float64
+    x = SI.real_uniform(0, N, dtype=rdt)
+    plan = F(N=N, P=P, B=B, Q=Q, precision=prec, direct=direct, real=True)
+    assert plan.info["N"] == N
+    y = plan(torch.from_numpy(x).cuda()).cpu().numpy()
+    assert y.shape == (N // 2 + 1,)
+    ref = O.rdft(x.astype(np.float64))
+    assert rel(y, ref) < TOL_E2E[prec]
+    # X_0 and X_{N/2} of a real input are real (up to rounding)
+    scale = np.sqrt(np.mean(np.abs(ref) ** 2))
+    assert abs(y[0].imag) < 10 * TOL_E2E[prec] * scale and abs(y[-1].imag) < 10 * TOL_E2E[prec] * scale
+    # end-to-end path with host buffers gives the same result
+    xh = torch.from_numpy(x).pin_memory()
+    oh = torch.empty(N // 2 + 1, dtype=plan.dtype).pin_memory()
+    plan.execute_host(xh, oh)
+    torch.cuda.synchronize()
+    assert rel(oh.numpy(), ref) < TOL_E2E[prec]
+
+
+def test_real_rejects_unsupported(F):
+    from paper_conf_sc_cecka17_b200._lib import FmmfftError
+    with pytest.raises(FmmfftError):
+        F(N=1 << 13, P=16, G=2, virtual=True, real=True)
+    with pytest.raises(FmmfftError):
+        F(N=1 << 13, P=16, inverse=True, real=True)
