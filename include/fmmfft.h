@@ -88,9 +88,16 @@ typedef enum {
                                    complex vector z_j = x_{2j} + i x_{2j+1}, transformed by the
                                    complex plan of length N/2 (P, B, Q, M_L — or DIRECT — apply
                                    to THAT length), then one elementwise pass (k_r2c_post)
-                                   separates the even / odd halves. G = 1 only, not with
-                                   INVERSE / VIRTUAL (else FMMFFT_UNSUPPORTED). fmmfft_get_info
-                                   reports the real N; M, L, ... describe the complex plan. */
+                                   separates the even / odd halves. With FMMFFT_FLAG_INVERSE:
+                                   the complex-to-real inverse x_j = (1/N) sum_{k<N} X_k
+                                   exp(+2 pi i jk/N) of a Hermitian spectrum given as X_0..X_{N/2}
+                                   (in = N/2 + 1 complex, out = N reals; the imaginary parts of
+                                   X_0 and X_{N/2} are ignored): one elementwise pass (k_c2r_pre)
+                                   builds the length-N/2 spectrum of z_j = x_{2j} + i x_{2j+1},
+                                   then the inverse complex plan writes z = the N reals in place.
+                                   G = 1 only, not with VIRTUAL (else FMMFFT_UNSUPPORTED).
+                                   fmmfft_get_info reports the real N; M, L, ... describe the
+                                   complex plan. */
 
 /* ---------------------------------------------------------------- communicator (G > 1)
  * One process per GPU. Rank 0 calls fmmfft_get_unique_id and broadcasts the 128 bytes (e.g.

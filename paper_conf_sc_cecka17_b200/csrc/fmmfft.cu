@@ -1331,6 +1331,16 @@ struct Exec {
 
     fmmfft_status_t run() {
         fmmfft_status_t st;
+        if (p->real && p->inverse) {                    // C2R: conj(Z) -> forward -> conj / H = z
+            const long long H = p->N;
+            C* Zc = (C*)p->ranks[0].cin;
+            const unsigned blocks = (unsigned)std::min<long long>((H / 2 + 256) / 256, 148LL * 8);
+            launch_pdl(k_c2r_pre<R>, blocks, 256, 0, s, in[0], Zc, H);
+            LAUNCH_CHECK();
+            in[0] = Zc;
+            if ((st = run_forward())) return st;
+            return conj_scale(out[0], out[0], R(1) / (R)H);
+        }
         if (p->real) {                                  // z_j = x_{2j} + i x_{2j+1}: the input as is
             C* X = out[0];
             out[0] = (C*)p->ranks[0].rz;
@@ -1773,8 +1783,7 @@ fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, i
     if (!plan) return fail(FMMFFT_INVALID_VALUE, "plan is NULL");
     *plan = nullptr;
     if (G != 1) return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_REAL: single GPU only (G = 1)");
-    if (flags & (FMMFFT_FLAG_INVERSE | FMMFFT_FLAG_VIRTUAL))
-        return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_REAL: forward, non-virtual plans only");
+    if (flags & FMMFFT_FLAG_VIRTUAL) return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_REAL: non-virtual plans only");
     if (N < 4 || (N & 1)) return fail(FMMFFT_INVALID_VALUE, "FMMFFT_FLAG_REAL: N must be even");
     fmmfft_status_t st = plan_complex(plan, N / 2, P, G, B, Q, precision, M_L, flags);
     if (st) return st;
@@ -1795,8 +1804,9 @@ fmmfft_status_t fmmfft_plan(fmmfft_plan_t* plan, long long N, int P, int G, int 
 fmmfft_status_t fmmfft_execute(fmmfft_plan_t p, const void* in, void* out, void* stream) {
     if (!p) return fail(FMMFFT_INVALID_VALUE, "plan is NULL");
     if (!in || !out) return fail(FMMFFT_INVALID_VALUE, "in/out is NULL");
-    const size_t bytes = (size_t)(p->virt ? p->N : p->N / p->G) * p->esz;
-    const size_t obytes = bytes + (p->real ? p->esz : 0);   // real plans: N/2 + 1 outputs
+    const size_t nb = (size_t)(p->virt ? p->N : p->N / p->G) * p->esz;
+    const size_t half = nb + (p->real ? p->esz : 0);        // real plans: N/2 + 1 complex values
+    const size_t bytes = p->real && p->inverse ? half : nb, obytes = p->real && p->inverse ? nb : half;
     const char* a = (const char*)in;
     const char* b = (const char*)out;
     if (a < b + obytes && b < a + bytes) return fail(FMMFFT_INVALID_VALUE, "in and out overlap");
@@ -1813,8 +1823,9 @@ fmmfft_status_t fmmfft_execute(fmmfft_plan_t p, const void* in, void* out, void*
 
 fmmfft_status_t fmmfft_execute_host(fmmfft_plan_t p, const void* in_host, void* out_host, void* stream) {
     if (!p || !in_host || !out_host) return fail(FMMFFT_INVALID_VALUE, "NULL argument");
-    const size_t bytes = (size_t)(p->virt ? p->N : p->N / p->G) * p->esz;
-    const size_t obytes = bytes + (p->real ? p->esz : 0);   // real plans: N/2 + 1 outputs
+    const size_t nb = (size_t)(p->virt ? p->N : p->N / p->G) * p->esz;
+    const size_t half = nb + (p->real ? p->esz : 0);        // real plans: N/2 + 1 complex values
+    const size_t bytes = p->real && p->inverse ? half : nb, obytes = p->real && p->inverse ? nb : half;
     RankBufs& rb = p->ranks[0];
     if (!rb.din) {
         fmmfft_status_t st;

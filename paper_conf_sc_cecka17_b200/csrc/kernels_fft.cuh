@@ -774,6 +774,43 @@ k_r2c_post(const C2<R>* __restrict__ Z, C2<R>* __restrict__ X, long long H) {
 }
 
 // ---------------------------------------------------------------------------------------------
+// k_c2r_pre (FMMFFT_FLAG_REAL | FMMFFT_FLAG_INVERSE): from X_k, k = 0..H, of a real signal of
+// length N = 2H (X_{N-k} = conj(X_k)), with a = X_k, b = conj(X_{H-k}):
+// E_k = (a + b)/2 and O_k = w_N^{-k} (a - b)/2 are the H-point spectra (scaled by 1/2) of the even
+// and odd samples, so z = F_H^{-1} Z with Z_k = E_k + i O_k is z_j = x_{2j} + i x_{2j+1}, i.e. the
+// N real outputs in place. Z_{H-k} = conj(E_k) + i conj(O_k). Writes conj(Z) (the inverse plan's
+// input conjugation, fused): thread k <= H/2 writes k and H - k (k = 0: only Z_0).
+// ---------------------------------------------------------------------------------------------
+template <typename R>
+__global__ void __launch_bounds__(256)
+k_c2r_pre(const C2<R>* __restrict__ X, C2<R>* __restrict__ Zc, long long H) {
+    pdl_trigger();
+    pdl_wait();
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    for (long long k = (long long)blockIdx.x * blockDim.x + threadIdx.x; k <= H / 2; k += stride) {
+        const C2<R> a = X[k];
+        const C2<R> xb = X[H - k];
+        const R Er = R(0.5) * (a.x + xb.x), Ei = R(0.5) * (a.y - xb.y);   // (a + conj(xb)) / 2
+        const R Dr = R(0.5) * (a.x - xb.x), Di = R(0.5) * (a.y + xb.y);   // (a - conj(xb)) / 2
+        R wr, wi;                                                        // w_N^{-k} = exp(+2 pi i k / 2H)
+        if constexpr (sizeof(R) == 4) {
+            float sn, cs;
+            sincospif((float)((double)k / (double)H), &sn, &cs);
+            wr = cs; wi = sn;
+        } else {
+            double sn, cs;
+            sincospi((double)k / (double)H, &sn, &cs);
+            wr = cs; wi = sn;
+        }
+        const R Or = wr * Dr - wi * Di, Oi = wr * Di + wi * Dr;            // O = w^{-k} D
+        // Z_k = E + i O = (Er - Oi) + i (Ei + Or); stored conjugated
+        Zc[k] = C2<R>{Er - Oi, -(Ei + Or)};
+        // Z_{H-k} = conj(E) + i conj(O) = (Er + Oi) + i (Or - Ei); stored conjugated
+        if (k != 0) Zc[H - k] = C2<R>{Er + Oi, Ei - Or};
+    }
+}
+
+// ---------------------------------------------------------------------------------------------
 // k_post_pfft_r: the same L2T + POST + P-point FFT + transposed store for P <= 32 with the whole
 // P-point column of one m in one thread's registers (no shared-memory FFT tile, no barriers in
 // the FFT): thread (box b, m) loads T_near[p][b][.][m] for all p (coalesced over m), adds

@@ -81,7 +81,10 @@ class FmmFFT:
                 (FLAG_INVERSE if inverse else 0) | (FLAG_DIRECT if direct else 0) | (FLAG_REAL if real else 0)
         self.inverse = inverse
         self.real = real
-        self.in_dtype = (torch.float32 if precision == "c64" else torch.float64) if real else self.dtype
+        rdt = torch.float32 if precision == "c64" else torch.float64
+        # real forward: N reals -> N/2+1 complex; real inverse: N/2+1 complex -> N reals
+        self.in_dtype = rdt if real and not inverse else self.dtype
+        self.out_dtype = rdt if real and inverse else self.dtype
         h = ctypes.c_void_p()
         check(lib.fmmfft_plan_ex(ctypes.byref(h), N, P, G, B, Q, self._prec, M_L, flags))
         self._h = h
@@ -89,13 +92,15 @@ class FmmFFT:
 
     # -- execution
     def __call__(self, x: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
-        if x.dtype != self.in_dtype or not x.is_cuda or not x.is_contiguous() or x.numel() != self.n_local:
-            raise ValueError(f"expected a contiguous CUDA {self.in_dtype} tensor of {self.n_local} elements")
-        n_out = self.N // 2 + 1 if self.real else self.n_local
+        half = self.N // 2 + 1
+        n_in = half if self.real and self.inverse else self.n_local
+        n_out = half if self.real and not self.inverse else self.n_local
+        if x.dtype != self.in_dtype or not x.is_cuda or not x.is_contiguous() or x.numel() != n_in:
+            raise ValueError(f"expected a contiguous CUDA {self.in_dtype} tensor of {n_in} elements")
         if out is None:
-            out = torch.empty(n_out, dtype=self.dtype, device=x.device)
-        elif out.dtype != self.dtype or not out.is_contiguous() or out.numel() != n_out:
-            raise ValueError(f"out must be a contiguous {self.dtype} tensor of {n_out} elements")
+            out = torch.empty(n_out, dtype=self.out_dtype, device=x.device)
+        elif out.dtype != self.out_dtype or not out.is_contiguous() or out.numel() != n_out:
+            raise ValueError(f"out must be a contiguous {self.out_dtype} tensor of {n_out} elements")
         check(lib.fmmfft_execute(self._h, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(out.data_ptr()),
                                  _stream_ptr(stream)))
         return out

@@ -367,4 +367,30 @@ def test_real_rejects_unsupported(F):
     with pytest.raises(FmmfftError):
         F(N=1 << 13, P=16, G=2, virtual=True, real=True)
     with pytest.raises(FmmfftError):
-        F(N=1 << 13, P=16, inverse=True, real=True)
+        F(N=1 << 13, P=16, G=2, virtual=True, inverse=True, real=True)
+
+
+@pytest.mark.parametrize("N,P,B,Q,prec,direct", [
+    (1 << 13, 16, 2, 16, "c128", False),
+    (1 << 13, 16, 2, 16, "c64", False),
+    (1 << 21, 64, 2, 16, "c64", False),
+    (1 << 21, 64, 2, 16, "c128", False),
+    (1 << 16, 1, 2, 16, "c64", True),
+    (1 << 16, 1, 2, 16, "c128", True),
+])
+def test_real_inverse_vs_oracle(F, N, P, B, Q, prec, direct):
+    # the spectrum of a seeded real signal, X_0..X_{N/2} (oracle rdft); the C2R inverse returns
+    # the signal: x = (1/N) sum_k X_k w_N^{-jk} with X_{N-k} = conj(X_k) (eq. 1 inverted)
+    rdt = np.float32 if prec == "c64" else np.float64
+    x = SI.real_uniform(0, N, dtype=np.float64)
+    X = O.rdft(x)
+    ref = np.real(O.fft_radix2(np.concatenate([X, np.conj(X[-2:0:-1])]), inverse=True))
+    assert np.max(np.abs(ref - x)) < 1e-12                      # the oracle round trip itself
+    inv = F(N=N, P=P, B=B, Q=Q, precision=prec, direct=direct, real=True, inverse=True)
+    y = inv(torch.from_numpy(X.astype(NPDT[prec])).cuda()).cpu().numpy()
+    assert y.dtype == rdt and y.shape == (N,)
+    assert np.linalg.norm(y - ref) / np.linalg.norm(ref) < TOL_E2E[prec]
+    # forward real plan -> inverse real plan round trip on the device
+    fwd = F(N=N, P=P, B=B, Q=Q, precision=prec, direct=direct, real=True)
+    z = inv(fwd(torch.from_numpy(x.astype(rdt)).cuda())).cpu().numpy()
+    assert np.linalg.norm(z - x) / np.linalg.norm(x) < 2 * TOL_E2E[prec]
