@@ -196,6 +196,37 @@ def cufft_comparator(x, flush, steps):
     return out
 
 
+def real_comparator(N, P, B, Q, prec, M_L, flush, steps):
+    """Context: the real-input transform (FMMFFT_FLAG_REAL) of 2N reals, whose
+    complex plan is this workload's (N, P, B, Q), against cuFFT's rfft (torch.fft.rfft) on the same
+    seeded input, same L2 flush and event timing. GFLOP/s use the real-FFT convention 2.5 n log2 n."""
+    import torch
+    import synth_inputs as SI
+    from paper_conf_sc_cecka17_b200 import FmmFFT
+    n = 2 * N
+    rdt = torch.float32 if prec == "c64" else torch.float64
+    xr = torch.from_numpy(SI.real_uniform(0, n)).to(rdt).cuda()
+    out = {"n_real": n, "flops_convention": "2.5 n log2 n"}
+    plan = FmmFFT(N=n, P=P, B=B, Q=Q, precision=prec, M_L=M_L, real=True)
+    y = torch.empty(N + 1, dtype=plan.dtype, device="cuda")
+    st = torch.cuda.current_stream()
+    for name, fn in (("fmmfft_r2c", lambda: plan(xr, y, st)), ("cufft_rfft", lambda: torch.fft.rfft(xr))):
+        for _ in range(3):
+            fn()
+        torch.cuda.synchronize()
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+        for a, b_ in ev:
+            flush.zero_()
+            a.record()
+            fn()
+            b_.record()
+        torch.cuda.synchronize()
+        ms = sum(a.elapsed_time(b_) for a, b_ in ev) / steps
+        out[name] = {"value": 2.5 * n * math.log2(n) / (ms * 1e-3) / 1e9, "unit": "GFLOP/s", "ms_per_step": ms}
+    plan.close()
+    return out
+
+
 # ------------------------------------------------------------------------------ CPU oracle legs
 def oracle_sample(workload: str, G: int, budget_s: float):
     """Time the CPU float64 oracle on a bounded sample of the workload: the full problem if one
@@ -433,6 +464,12 @@ def run_fmmfft(args, rank, world, local_rank):
                          "note": "fmmfft_autotune pick for the same N / precision / error bound; context, not the headline"}
         except Exception as e:
             autotuned = {"error": str(e)[:200]}
+    real_ctx = None
+    if world == 1 and not args.no_extras and vg == 1:
+        try:
+            real_ctx = real_comparator(N, P, B, Q, prec, M_L, flush, min(args.steps, 50))
+        except Exception as e:  # context only
+            real_ctx = {"error": str(e)[:200]}
     if rank != 0:
         return
     peaks = load_peaks()
@@ -493,6 +530,7 @@ def run_fmmfft(args, rank, world, local_rank):
     if world == 1:
         line["comparator"] = cufft_comp
         line["autotuned"] = autotuned
+        line["real_input"] = real_ctx
     if world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(workload, G)
     print(json.dumps(line), flush=True)
