@@ -202,27 +202,52 @@ def test_profile_stage_times(F):
 
 
 # ------------------------------------------------------------------ full-size bench configs, sampled
-def sampled_dft(x, ks):
+def sampled_dft(x, ks, chunk=1 << 24):
+    """y_k of eq. (1) one k at a time (exact integer j*k mod N), in chunks of j to bound memory."""
     N = len(x)
-    j = np.arange(N, dtype=np.int64)
-    xc = x.astype(np.complex128)
-    return np.array([np.dot(xc, np.exp(-2j * np.pi * ((j * k) % N) / N)) for k in ks])
+    out = []
+    for k in ks:
+        acc = 0j
+        for a in range(0, N, chunk):
+            j = np.arange(a, min(N, a + chunk), dtype=np.int64)
+            acc += np.dot(x[a:a + len(j)].astype(np.complex128), np.exp(-2j * np.pi * ((j * int(k)) % N) / N))
+        out.append(acc)
+    return np.array(out)
 
 
 @pytest.mark.parametrize("N,P,B,Q,prec,G", [
     (1 << 20, 64, 2, 16, "c64", 1),      # cfg2 — exactly the bench.py N=1 launch configuration
     (1 << 26, 128, 4, 16, "c64", 8),     # cfg3 shape (G = 8) as virtual ranks on one GPU
+    (1 << 28, 64, 2, 24, "c128", 1),     # cfg4 (N = 2^28 complex128, Q = 24) on one GPU
 ])
 def test_full_size_sampled(F, N, P, B, Q, prec, G):
     plan, x, y = run(F, N, P, B, Q, prec, 64, G=G, virtual=G > 1)
+    plan.close()
     rng = np.random.default_rng(0)
     ks = np.concatenate([[0, 1, N // 2, N - 1], rng.integers(0, N, 8)])
     ref = sampled_dft(x, ks)
-    assert np.linalg.norm(y[ks] - ref) / np.linalg.norm(ref) < 1e-5
+    assert np.linalg.norm(y[ks] - ref) / np.linalg.norm(ref) < TOL_E2E[prec]
     # Parseval holds at any size: ||y||^2 = N ||x||^2
     ny = np.sum(np.abs(y.astype(np.complex128)) ** 2)
     nx = np.sum(np.abs(x.astype(np.complex128)) ** 2)
-    assert abs(ny / (N * nx) - 1) < 1e-5
+    assert abs(ny / (N * nx) - 1) < TOL_E2E[prec]
+
+
+def test_real_full_size_sampled(F):
+    # 2^27 reals: the complex plan is cfg3's shape at G = 1 (N/2 = 2^26, P = 16, B = 4, Q = 16)
+    N = 1 << 27
+    x = SI.real_uniform(0, N, dtype=np.float32)
+    plan = F(N=N, P=16, B=4, Q=16, precision="c64", real=True)
+    y = plan(torch.from_numpy(x).cuda()).cpu().numpy()
+    plan.close()
+    rng = np.random.default_rng(1)
+    ks = np.concatenate([[0, 1, N // 4, N // 2 - 1, N // 2], rng.integers(0, N // 2 + 1, 7)])
+    ref = sampled_dft(x, ks)
+    assert np.linalg.norm(y[ks] - ref) / np.linalg.norm(ref) < 1e-5
+    # Parseval for a real signal: |X_0|^2 + |X_{N/2}|^2 + 2 sum_{0<k<N/2} |X_k|^2 = N ||x||^2
+    a = np.abs(y.astype(np.complex128)) ** 2
+    ny = a[0] + a[-1] + 2 * np.sum(a[1:-1])
+    assert abs(ny / (N * np.sum(x.astype(np.float64) ** 2)) - 1) < 1e-5
 
 
 # ------------------------------------------------------------------ alternative kernel paths
