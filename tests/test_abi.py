@@ -51,6 +51,7 @@ def test_version_and_last_error(L):
     ((1 << 20, 64, 1, 2, 16, 0, 8, 0), b"M_L"),                 # M_L = 8 < 16
     ((1 << 20, 4, 8, 2, 16, 0, 64, 1), b"P % G"),               # P % G != 0
     ((1 << 20, 64, 2, 2, 16, 0, 64, 0), b"fmmfft_comm_init"),   # G > 1 without a communicator
+    ((1001, 16, 1, 2, 16, 0, 64, 32), b"even"),                 # FMMFFT_FLAG_REAL with odd N
 ])
 def test_invalid_plans_rejected(L, args, frag):
     h = ctypes.c_void_p()
@@ -98,3 +99,17 @@ def test_autotune_model_host_only():
         autotune(1 << 20, precision="c64", tol=1e-8, measure=False)      # below the fp32 floor
     with pytest.raises(FmmfftError):
         autotune(1 << 20, G=2, precision="c64", measure=True)           # measuring is G = 1 only
+
+
+def test_flag_values_match_header(L):
+    src = open(os.path.join(ROOT, "include", "fmmfft.h")).read()
+    hdr = {m[0]: int(m[1]) for m in re.findall(r"#define FMMFFT_FLAG_(\w+)\s+(\d+)u", src)}
+    assert hdr == {"VIRTUAL": L.FLAG_VIRTUAL, "PROFILE": L.FLAG_PROFILE, "DEBUG": L.FLAG_DEBUG,
+                   "INVERSE": L.FLAG_INVERSE, "DIRECT": L.FLAG_DIRECT, "REAL": L.FLAG_REAL}
+
+
+def test_real_multi_gpu_unsupported(L):
+    # FMMFFT_FLAG_REAL is single-GPU: rejected before any device or communicator is touched
+    h = ctypes.c_void_p()
+    st = L.lib.fmmfft_plan_ex(ctypes.byref(h), 1 << 21, 64, 2, 2, 16, 0, 64, 32 | 1)
+    assert st == L.UNSUPPORTED and b"G = 1" in L.lib.fmmfft_last_error() and not h.value
