@@ -347,6 +347,16 @@ def test_autotune_measured_meets_tol(F):
     assert rel(y, O.fft_radix2(x)) < 1e-5
 
 
+@pytest.mark.parametrize("N", [1 << 20, 1 << 22])
+def test_autotune_c128_meets_tol(F, N):
+    # the complex128 pick (Q from the error model, e.g. Q = 16 instead of cfg4's Q = 24) must still
+    # meet the north star's 1e-11 bound against the float64 FFT
+    from paper_conf_sc_cecka17_b200 import autotune
+    t = autotune(N, G=1, precision="c128", tol=1e-11, measure=False)
+    plan, x, y = run(F, N, t["P"], t["B"], t["Q"], "c128", t["M_L"])
+    assert rel(y, O.fft_radix2(x)) < 1e-11
+
+
 @pytest.mark.parametrize("env", [None, {"FMMFFT_PP": "tile"}])
 @pytest.mark.parametrize("P,Q,prec", [(16, 16, "c64"), (32, 8, "c64"), (8, 24, "c128"), (2, 16, "c64"), (64, 16, "c64"), (64, 24, "c128")])
 def test_post_pfft_variants(F, monkeypatch, env, P, Q, prec):
