@@ -63,6 +63,12 @@ typedef enum {
                                    runs with device-to-device copies instead of NCCL. in/out
                                    are then the FULL length-N vectors. For testing the
                                    partitioned algorithm on one GPU. */
+#define FMMFFT_FLAG_VIRTUAL_NCCL 64u  /* with FMMFFT_FLAG_VIRTUAL: the virtual ranks' exchanges go
+                                   through NCCL (ncclSend / ncclRecv to self, ncclGroupStart/End,
+                                   captured in the execute graph) on a 1-rank communicator
+                                   (fmmfft_comm_init(0, 1, id) on this device) instead of device
+                                   copies — the NCCL transport on one GPU (else NOT_INITIALIZED
+                                   / INVALID_VALUE). */
 #define FMMFFT_FLAG_PROFILE 2u  /* record CUDA events around every stage (fmmfft_stage_times) */
 #define FMMFFT_FLAG_DEBUG 4u    /* keep every level's M^l / L^l in the buffers fmmfft_debug_buffer
                                    returns. Without it the fused single-GPU far field
@@ -106,7 +112,8 @@ typedef enum {
  * at run time (dlopen "libnccl.so.2"); FMMFFT_NCCL_ERROR if it cannot be found. */
 FMMFFT_API fmmfft_status_t fmmfft_get_unique_id(unsigned char id[128]);
 FMMFFT_API fmmfft_status_t fmmfft_comm_init(int rank, int G, const unsigned char id[128]);
-FMMFFT_API fmmfft_status_t fmmfft_comm_destroy(void);
+FMMFFT_API fmmfft_status_t fmmfft_comm_destroy(void);  /* INVALID_VALUE while a plan created on the
+                                                           communicator is alive */
 
 /* ---------------------------------------------------------------- plans
  * fmmfft_plan: N = M P points, P FMMs interleaved (P - 1 non-trivial), G ranks, base level
@@ -192,8 +199,10 @@ FMMFFT_API fmmfft_status_t fmmfft_get_info(fmmfft_plan_t plan, fmmfft_info_t* in
 /* Per-stage device times (ms) of the LAST execute of a plan created with
  * FMMFFT_FLAG_PROFILE (else INVALID_VALUE); synchronises that execute's stream. Stage i's
  * name is fmmfft_stage_name(i): comm_S, s2m, m2m, comm_M, top, down, post_pfft, a2a, mfft —
- * consecutive intervals of the main stream — and s2t, the near field on the side stream that
- * overlaps s2m..down. n = capacity of ms[]; returns the count in *n_out. */
+ * consecutive intervals of the stream — and s2t, the near field. A profiled plan runs the near
+ * field (S halo + S2T) serialised on the main stream instead of concurrently on its side
+ * stream, so each interval holds only its own kernels (s2m excludes the S2T that follows it).
+ * n = capacity of ms[]; returns the count in *n_out. */
 FMMFFT_API fmmfft_status_t fmmfft_stage_times(fmmfft_plan_t plan, float* ms, int n, int* n_out);
 FMMFFT_API const char* fmmfft_stage_name(int i);
 

@@ -3,7 +3,7 @@ Edelman factorisation F_N = F_{M,P} H^_{M,P}, with sm_100a CUDA kernels behind t
 include/fmmfft.h. The CUDA library is required — there is no CPU fallback: touching FmmFFT
 (or init_comm / destroy_comm) raises ImportError if libfmmfft.so is missing."""
 
-__all__ = ["FmmFFT", "init_comm", "destroy_comm", "autotune"]
+__all__ = ["FmmFFT", "init_comm", "init_comm_local", "destroy_comm", "autotune"]
 
 
 def __getattr__(name):  # lazy, so `python -m paper_conf_sc_cecka17_b200.build` works unbuilt

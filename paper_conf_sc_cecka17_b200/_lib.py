@@ -13,7 +13,7 @@ SUCCESS, INVALID_VALUE, UNSUPPORTED, ALLOC_FAILED, CUDA_ERROR, NCCL_ERROR, NOT_I
 STATUS_NAMES = ["SUCCESS", "INVALID_VALUE", "UNSUPPORTED", "ALLOC_FAILED", "CUDA_ERROR", "NCCL_ERROR",
                 "NOT_INITIALIZED"]
 C64, C128 = 0, 1
-FLAG_VIRTUAL, FLAG_PROFILE, FLAG_DEBUG, FLAG_INVERSE, FLAG_DIRECT, FLAG_REAL = 1, 2, 4, 8, 16, 32
+FLAG_VIRTUAL, FLAG_PROFILE, FLAG_DEBUG, FLAG_INVERSE, FLAG_DIRECT, FLAG_REAL, FLAG_VIRTUAL_NCCL = 1, 2, 4, 8, 16, 32, 64
 
 # every symbol include/fmmfft.h declares (checked by tests/test_abi.py)
 EXPORTS = [

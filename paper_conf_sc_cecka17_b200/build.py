@@ -53,7 +53,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not needs_build():
         return LIB
     cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
-           "-Xcompiler", "-fvisibility=hidden", "--expt-relaxed-constexpr",
+           "-Xcompiler", "-fvisibility=hidden", "--expt-relaxed-constexpr", "--split-compile=8",
            "-I", os.path.join(ROOT, "include"), "-I", _nccl_include(),
            os.path.join(CSRC, "fmmfft.cu"), "-o", LIB + ".tmp", "-ldl"]
     if verbose:
@@ -64,6 +64,22 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB
 
 
+CMP_SRC = os.path.join(ROOT, "comparators", "cufftxt.cu")
+CMP_LIB = os.path.join(ROOT, "comparators", "libcufftxt_cmp.so")
+
+
+def build_comparator(force: bool = False) -> str:
+    """The cuFFTXt comparator (comparators/cufftxt.cu, a library call timed by bench.py at G > 1;
+    not part of the product path)."""
+    if not force and os.path.exists(CMP_LIB) and os.path.getmtime(CMP_LIB) >= os.path.getmtime(CMP_SRC):
+        return CMP_LIB
+    subprocess.run([_nvcc(), *ARCH, "-O2", "-shared", "-Xcompiler", "-fPIC", CMP_SRC, "-o", CMP_LIB + ".tmp", "-lcufft"],
+                   check=True)
+    os.replace(CMP_LIB + ".tmp", CMP_LIB)
+    return CMP_LIB
+
+
 if __name__ == "__main__":
     build(force="--force" in sys.argv, verbose="-v" in sys.argv)
+    build_comparator(force="--force" in sys.argv)
     print(LIB)

@@ -26,6 +26,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <atomic>
 #include <mutex>
 #include <string>
 #include <type_traits>
@@ -137,12 +138,34 @@ static cudaError_t launch_cluster(void (*kern)(KArgs...), dim3 grid, dim3 block,
     return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
 }
 
+// makes `dev` current for a scope, restoring the caller's device on exit
+struct DeviceGuard {
+    int prev = -1;
+    cudaError_t err = cudaSuccess;
+    explicit DeviceGuard(int dev) {
+        err = cudaGetDevice(&prev);
+        if (err == cudaSuccess && prev != dev) err = cudaSetDevice(dev);
+        else prev = -1;
+    }
+    ~DeviceGuard() { if (prev >= 0) cudaSetDevice(prev); }
+};
+
 // ------------------------------------------------------------------ communicator
 struct Comm {
     ncclComm_t comm = nullptr;
     int rank = 0, size = 0, device = -1;
 };
 static Comm g_comm;
+static std::atomic<int> g_comm_plans{0};    // live plans holding g_comm.comm (comm_destroy refuses)
+
+// One point-to-point transfer of a rank's exchange, exactly the arguments of its ncclSend /
+// ncclRecv (n complex elements). Every exchange (S halo, M^l halos, the all-to-all) is first
+// written as the per-rank list of these; NCCL plans issue their own rank's list in one group,
+// virtual plans execute every rank's list by matching the k-th send g -> q with the k-th receive
+// at q from g (NCCL's in-order matching per peer pair), so the virtual data flow exercises the
+// very pointer and count arithmetic the NCCL branch issues.
+struct P2P { bool send; int peer; void* ptr; size_t n; };
+struct Gather { const void* send; void* recv; size_t n; };    // ncclAllGather(send, recv, n)
 
 // ------------------------------------------------------------------ host operator tables (fp64)
 // These are the product's own tables (computed here in C++); they share nothing with oracle/.
@@ -237,6 +260,11 @@ struct fmmfft_plan_s {
     cudaEvent_t fork = nullptr, join = nullptr;   // side-stream fork / join
     cudaEvent_t fork2 = nullptr;     // S' ready (tensor-core S2T)
     cudaStream_t side = nullptr;     // S2T runs here, concurrently with the far field
+    cudaEvent_t cs_done = nullptr;   // S halo exchange (side stream) complete: orders NCCL work
+    ncclComm_t comm = nullptr;       // G > 1 (non-virtual): the communicator, bound at plan time;
+                                     // virtual + FMMFFT_FLAG_VIRTUAL_NCCL: a 1-rank communicator
+    int comm_rank = 0;
+    bool vnccl = false;              // virtual ranks exchange through NCCL self send / recv
     bool have_times = false;
     bool use_graph = true;
     cudaStream_t cap_stream = nullptr;
@@ -472,17 +500,25 @@ static void destroy_plan(fmmfft_plan_s* p) {
     if (p->fork) cudaEventDestroy(p->fork);
     if (p->join) cudaEventDestroy(p->join);
     if (p->fork2) cudaEventDestroy(p->fork2);
+    if (p->cs_done) cudaEventDestroy(p->cs_done);
+    if (p->comm) --g_comm_plans;
     if (p->side) cudaStreamDestroy(p->side);
     if (p->cap_stream) cudaStreamDestroy(p->cap_stream);
     delete p;
 }
 
-// Raise every kernel's dynamic shared memory cap once per process (not legal during capture).
+// Raise every kernel's dynamic shared memory cap once per device (function attributes are
+// per device; not legal during capture). Called with the plan's device current.
 template <typename R>
 static fmmfft_status_t init_kernel_attrs() {
-    static std::once_flag once;
-    static cudaError_t err = cudaSuccess;
-    std::call_once(once, [] {
+    constexpr int kMaxDev = 64;
+    static std::once_flag once_dev[kMaxDev];
+    static cudaError_t err_dev[kMaxDev] = {};
+    int cur = 0;
+    CUDA_TRY(cudaGetDevice(&cur));
+    if (cur < 0 || cur >= kMaxDev) return fail(FMMFFT_UNSUPPORTED, "device ordinal %d", cur);
+    cudaError_t& err = err_dev[cur];
+    std::call_once(once_dev[cur], [&err] {
         int dev = 0, optin = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
@@ -617,12 +653,17 @@ struct Exec {
     int nb_at(int lev) const { return (int)((1LL << lev) / p->G); }
     C* interior(void* pad) const { return (C*)pad + 2 * QP(); }
     ncclDataType_t nt() const { return sizeof(R) == 4 ? ncclFloat : ncclDouble; }
-    int grank(const RankBufs& rb) const { return p->virt ? rb.g : (p->G > 1 ? g_comm.rank : 0); }
+    int grank(const RankBufs& rb) const { return p->virt ? rb.g : p->comm_rank; }
 
     template <typename F> bool with_pcd(F&& f) const {
         if constexpr (sizeof(R) == 4) return dispatch<2, 4, 8, 16>(p->PCd, f);
         else return dispatch<2, 4, 8>(p->PCd, f);
     }
+
+    // the stream of the near field (S halo + S2T): concurrent with the far field, except in
+    // profiled plans, which serialise it on the main stream so every stage's events bracket only
+    // its own kernels (fmmfft_stage_times: s2t measured alone, s2m excludes it)
+    cudaStream_t side() const { return (p->flags & FMMFFT_FLAG_PROFILE) ? s : p->side; }
 
     // stage boundary event; inside a graph capture it must be an "external" record to become a
     // real event-record node (a plain record during capture only expresses a dependency)
@@ -632,31 +673,132 @@ struct Exec {
         return FMMFFT_SUCCESS;
     }
 
-    // ---- comm_S: S halo (line 2)
-    fmmfft_status_t comm_S() {
-        if (p->G == 1) return FMMFFT_SUCCESS;
+    // ---- the exchanges, written once per rank as the NCCL arguments (P2P lists) --------------
+    int gidx(const RankBufs& rb) const { return p->virt ? rb.g : 0; }   // index into in[] / out[]
+
+    // S halo (line 2): rank g sends its box 0 to the left neighbour (whose right halo it
+    // is) and its last box to the right one; receives haloR from the right, haloL from the left
+    std::vector<P2P> sched_S(const RankBufs& rb) const {
         const size_t box = (size_t)p->M_L * p->P;
-        const int G = p->G;
-        if (p->virt) {
-            for (int g = 0; g < G; ++g) {
-                RankBufs& rb = p->ranks[g];
-                const C* left = in[(g - 1 + G) % G];
-                const C* right = in[(g + 1) % G];
-                CUDA_TRY(cudaMemcpyAsync(rb.haloL, left + (size_t)(p->nb - 1) * box, box * sizeof(C), cudaMemcpyDeviceToDevice, s));
-                CUDA_TRY(cudaMemcpyAsync(rb.haloR, right, box * sizeof(C), cudaMemcpyDeviceToDevice, s));
+        const int G = p->G, g = grank(rb), lf = (g - 1 + G) % G, rt = (g + 1) % G;
+        C* S = const_cast<C*>(in[gidx(rb)]);
+        return {{true, lf, S, box}, {true, rt, S + (size_t)(p->nb - 1) * box, box},
+                {false, rt, rb.haloR, box}, {false, lf, rb.haloL, box}};
+    }
+
+    // M^l halos for l > l_g (line 7): two boxes per side per level, all levels in one
+    // group; Mpad[l] = [2 left halo | nbl own | 2 right halo] boxes of Q P each
+    std::vector<P2P> sched_M(const RankBufs& rb) const {
+        const size_t QPc = QP();
+        const int G = p->G, g = grank(rb), lf = (g - 1 + G) % G, rt = (g + 1) % G;
+        std::vector<P2P> v;
+        for (int lev = p->lg + 1; lev <= p->L; ++lev) {
+            const size_t nbl = (size_t)nb_at(lev);
+            C* pad = (C*)rb.Mpad[lev];
+            v.push_back({true, lf, pad + 2 * QPc, 2 * QPc});              // own boxes 0, 1 -> left
+            v.push_back({true, rt, pad + nbl * QPc, 2 * QPc});            // own boxes nbl-2, nbl-1 -> right
+            v.push_back({false, rt, pad + (nbl + 2) * QPc, 2 * QPc});
+            v.push_back({false, lf, pad, 2 * QPc});
+        }
+        return v;
+    }
+
+    // all-gather of level l_g (line 9 / reading R16)
+    Gather sched_gather(const RankBufs& rb) const {
+        return {interior(rb.Mpad[p->lg]), rb.Mfull[p->lg], (size_t)nb_at(p->lg) * QP()};
+    }
+
+    // the one all-to-all (line 16): chunk r of W (k2 in r's block, own m) -> rank r's
+    // receive slot g
+    std::vector<P2P> sched_A2A(const RankBufs& rb) const {
+        const size_t chunk = (size_t)(p->P / p->G) * p->Mg;
+        std::vector<P2P> v;
+        for (int r = 0; r < p->G; ++r) {
+            v.push_back({true, r, (C*)rb.W + r * chunk, chunk});
+            v.push_back({false, r, (C*)rb.Rcv + r * chunk, chunk});
+        }
+        return v;
+    }
+
+    // issue one exchange on stream st: NCCL group (one process per GPU), or every virtual rank's
+    // list matched send-to-receive and executed as device copies (or NCCL self send / receive on
+    // a 1-rank communicator, FMMFFT_FLAG_VIRTUAL_NCCL)
+    template <typename Sched>
+    fmmfft_status_t exchange(Sched sched, cudaStream_t st) {
+        NcclApi& n = nccl();
+        if (!p->virt) {
+            const std::vector<P2P> v = sched(p->ranks[0]);
+            NCCL_TRY(n.GroupStart());
+            for (const P2P& o : v) {
+                if (o.send) NCCL_TRY(n.Send(o.ptr, 2 * o.n, nt(), o.peer, p->comm, st));
+                else        NCCL_TRY(n.Recv(o.ptr, 2 * o.n, nt(), o.peer, p->comm, st));
             }
+            NCCL_TRY(n.GroupEnd());
             return FMMFFT_SUCCESS;
         }
-        RankBufs& rb = p->ranks[0];
-        const int g = g_comm.rank, lf = (g - 1 + G) % G, rt = (g + 1) % G;
-        NcclApi& n = nccl();
-        NCCL_TRY(n.GroupStart());
-        NCCL_TRY(n.Send(in[0], 2 * box, nt(), lf, g_comm.comm, s));
-        NCCL_TRY(n.Send(in[0] + (size_t)(p->nb - 1) * box, 2 * box, nt(), rt, g_comm.comm, s));
-        NCCL_TRY(n.Recv(rb.haloR, 2 * box, nt(), rt, g_comm.comm, s));
-        NCCL_TRY(n.Recv(rb.haloL, 2 * box, nt(), lf, g_comm.comm, s));
-        NCCL_TRY(n.GroupEnd());
+        const int G = p->G;
+        std::vector<std::vector<P2P>> all(G);
+        for (RankBufs& rb : p->ranks) all[rb.g] = sched(rb);
+        std::vector<size_t> cur((size_t)G * G, 0);            // (receiver, sender) -> next receive op
+        std::vector<std::pair<const P2P*, const P2P*>> pairs;
+        for (int g = 0; g < G; ++g)
+            for (const P2P& o : all[g]) {
+                if (!o.send) continue;
+                const std::vector<P2P>& rv = all[o.peer];
+                size_t& k = cur[(size_t)o.peer * G + g];
+                while (k < rv.size() && (rv[k].send || rv[k].peer != g)) ++k;
+                if (k == rv.size()) return fail(FMMFFT_INVALID_VALUE, "exchange: send %d->%d has no receive", g, o.peer);
+                if (rv[k].n != o.n) return fail(FMMFFT_INVALID_VALUE, "exchange: %d->%d sends %zu, receives %zu", g, o.peer, o.n, rv[k].n);
+                pairs.push_back({&o, &rv[k]});
+                ++k;
+            }
+        size_t nrecv = 0;
+        for (auto& v : all) for (const P2P& o : v) nrecv += !o.send;
+        if (nrecv != pairs.size()) return fail(FMMFFT_INVALID_VALUE, "exchange: %zu receives, %zu sends", nrecv, pairs.size());
+        if (p->vnccl) {
+            NCCL_TRY(n.GroupStart());
+            for (auto& pr : pairs) {
+                NCCL_TRY(n.Send(pr.first->ptr, 2 * pr.first->n, nt(), 0, p->comm, st));
+                NCCL_TRY(n.Recv(pr.second->ptr, 2 * pr.second->n, nt(), 0, p->comm, st));
+            }
+            NCCL_TRY(n.GroupEnd());
+            return FMMFFT_SUCCESS;
+        }
+        for (auto& pr : pairs)
+            CUDA_TRY(cudaMemcpyAsync(pr.second->ptr, pr.first->ptr, pr.first->n * sizeof(C), cudaMemcpyDeviceToDevice, st));
         return FMMFFT_SUCCESS;
+    }
+
+    fmmfft_status_t allgather(cudaStream_t st) {
+        NcclApi& n = nccl();
+        if (!p->virt) {
+            const Gather a = sched_gather(p->ranks[0]);
+            NCCL_TRY(n.AllGather(a.send, a.recv, 2 * a.n, nt(), p->comm, st));
+            return FMMFFT_SUCCESS;
+        }
+        if (p->vnccl) NCCL_TRY(n.GroupStart());
+        for (RankBufs& dst : p->ranks) {
+            const Gather d = sched_gather(dst);
+            for (RankBufs& src : p->ranks) {
+                const Gather a = sched_gather(src);
+                if (a.n != d.n) return fail(FMMFFT_INVALID_VALUE, "allgather: counts differ");
+                C* to = (C*)d.recv + (size_t)src.g * a.n;
+                if (p->vnccl) {
+                    NCCL_TRY(n.Send(a.send, 2 * a.n, nt(), 0, p->comm, st));
+                    NCCL_TRY(n.Recv(to, 2 * a.n, nt(), 0, p->comm, st));
+                } else {
+                    CUDA_TRY(cudaMemcpyAsync(to, a.send, a.n * sizeof(C), cudaMemcpyDeviceToDevice, st));
+                }
+            }
+        }
+        if (p->vnccl) NCCL_TRY(n.GroupEnd());
+        return FMMFFT_SUCCESS;
+    }
+
+    // ---- comm_S: S halo (line 2) on the side stream, ahead of S2T (overlaps S2M)
+    fmmfft_status_t comm_S(cudaStream_t st) {
+        if (p->G == 1) return FMMFFT_SUCCESS;
+        return exchange([this](const RankBufs& rb) { return sched_S(rb); }, st);
     }
 
     // record a stage-boundary-style event on an arbitrary stream (S2T's own pair)
@@ -689,15 +831,13 @@ struct Exec {
             });
             LAUNCH_CHECK();
         }
-        // fork after S2M (so S2M runs alone): S2T on the side stream
-        CUDA_TRY(cudaEventRecord(p->fork, s));
-        CUDA_TRY(cudaStreamWaitEvent(p->side, p->fork, 0));
-        if ((st = mark_on(p->ev_s2t[0], p->side))) return st;
+        // fork after S2M (so S2M runs alone; the tensor-core S2T needs its S'): S2T on the side
+        // stream, behind the S halo exchange already queued there (G > 1)
+        CUDA_TRY(cudaEventRecord(p->fork2, s));
+        CUDA_TRY(cudaStreamWaitEvent(side(), p->fork2, 0));
+        if ((st = mark_on(p->ev_s2t[0], side()))) return st;
         if constexpr (sizeof(R) == 4) {
             if (p->s2t_tc) {                                   // tensor cores (tcgen05, 3xTF32)
-                CUDA_TRY(cudaEventRecord(p->fork2, s));             // needs S' from k_s2m
-                CUDA_TRY(cudaStreamWaitEvent(p->side, p->fork2, 0));
-                if ((st = mark_on(p->ev_s2t[0], p->side))) return st;
                 const int ntile = p->nb / S2TC_BOXES;
                 // tiles per CTA: the fewest that keep the grid within one wave of 148 SMs
                 // (one CTA per SM: TMEM + ~180 KB of shared memory)
@@ -709,15 +849,15 @@ struct Exec {
                     // several tiles per CTA: A chunks prefetched two ahead; one tile: one ahead (the
                     // first chunk's loads alone, so the first MMAs start sooner)
                     if (tpc > 1)
-                        launch_pdl(k_s2t_tc<2>, grid, S2TC_THREADS, s2tc_smem_bytes(), p->side, (const C*)rb.Sp, (const C*)rb.haloL,
+                        launch_pdl(k_s2t_tc<2>, grid, S2TC_THREADS, s2tc_smem_bytes(), side(), (const C*)rb.Sp, (const C*)rb.haloL,
                                    (const C*)rb.haloR, (float*)rb.Tn, (const float*)p->toep, p->P, p->nb, p->G, tpc);
                     else
-                        launch_pdl(k_s2t_tc<1>, grid, S2TC_THREADS, s2tc_smem_bytes(), p->side, (const C*)rb.Sp, (const C*)rb.haloL,
+                        launch_pdl(k_s2t_tc<1>, grid, S2TC_THREADS, s2tc_smem_bytes(), side(), (const C*)rb.Sp, (const C*)rb.haloL,
                                    (const C*)rb.haloR, (float*)rb.Tn, (const float*)p->toep, p->P, p->nb, p->G, tpc);
                     LAUNCH_CHECK();
                 }
-                if ((st = mark_on(p->ev_s2t[1], p->side))) return st;
-                CUDA_TRY(cudaEventRecord(p->join, p->side));
+                if ((st = mark_on(p->ev_s2t[1], side()))) return st;
+                CUDA_TRY(cudaEventRecord(p->join, side()));
                 return FMMFFT_SUCCESS;
             }
         }
@@ -738,15 +878,15 @@ struct Exec {
                 constexpr int PCv = decltype(pc)::value;
                 if constexpr (sizeof(R) == 8 && PCv > 16) return;
                 else
-                    launch_pdl(k_near_up<R, IB, PCv>, grid, threads, smem, p->side, S, hl, hr, (C*)rb.Tn, nullptr,
+                    launch_pdl(k_near_up<R, IB, PCv>, grid, threads, smem, side(), S, hl, hr, (C*)rb.Tn, nullptr,
                                                                             (const R*)p->s2t, p->s2t_chunk, (const R*)p->s2m,
                                                                             p->P, p->M_L, p->Q, p->nb, bpc);
             };
             dispatch<2, 4, 8, 16, 32>(PC_, go);
             LAUNCH_CHECK();
         }
-        if ((st = mark_on(p->ev_s2t[1], p->side))) return st;
-        CUDA_TRY(cudaEventRecord(p->join, p->side));
+        if ((st = mark_on(p->ev_s2t[1], side()))) return st;
+        CUDA_TRY(cudaEventRecord(p->join, side()));
         return FMMFFT_SUCCESS;
     }
 
@@ -910,40 +1050,11 @@ struct Exec {
     // ---- comm_M: halos (2 boxes per side) for l in (l_g, L] and all-gather of level l_g
     fmmfft_status_t comm_M() {
         if (p->G == 1) return FMMFFT_SUCCESS;
-        const size_t QPc = QP();
-        const int G = p->G;
-        const long long nlg = nb_at(p->lg);
-        if (p->virt) {
-            for (int g = 0; g < G; ++g) {
-                RankBufs& rb = p->ranks[g];
-                RankBufs& lf = p->ranks[(g - 1 + G) % G];
-                RankBufs& rt = p->ranks[(g + 1) % G];
-                for (int lev = p->lg + 1; lev <= p->L; ++lev) {
-                    const int nbl = nb_at(lev);
-                    CUDA_TRY(cudaMemcpyAsync(rb.Mpad[lev], (C*)lf.Mpad[lev] + (size_t)nbl * QPc, 2 * QPc * sizeof(C), cudaMemcpyDeviceToDevice, s));
-                    CUDA_TRY(cudaMemcpyAsync((C*)rb.Mpad[lev] + (size_t)(nbl + 2) * QPc, (C*)rt.Mpad[lev] + 2 * QPc, 2 * QPc * sizeof(C), cudaMemcpyDeviceToDevice, s));
-                }
-                for (int src = 0; src < G; ++src)
-                    CUDA_TRY(cudaMemcpyAsync((C*)rb.Mfull[p->lg] + (size_t)src * nlg * QPc, interior(p->ranks[src].Mpad[p->lg]),
-                                             nlg * QPc * sizeof(C), cudaMemcpyDeviceToDevice, s));
-            }
-            return FMMFFT_SUCCESS;
-        }
-        RankBufs& rb = p->ranks[0];
-        const int g = g_comm.rank, lf = (g - 1 + G) % G, rt = (g + 1) % G;
-        NcclApi& n = nccl();
-        NCCL_TRY(n.GroupStart());
-        for (int lev = p->lg + 1; lev <= p->L; ++lev) {
-            const int nbl = nb_at(lev);
-            C* pad = (C*)rb.Mpad[lev];
-            NCCL_TRY(n.Send(pad + 2 * QPc, 4 * QPc, nt(), lf, g_comm.comm, s));              // own boxes 0,1 -> left
-            NCCL_TRY(n.Send(pad + (size_t)nbl * QPc, 4 * QPc, nt(), rt, g_comm.comm, s));    // own boxes nb-2, nb-1 -> right
-            NCCL_TRY(n.Recv(pad + (size_t)(nbl + 2) * QPc, 4 * QPc, nt(), rt, g_comm.comm, s));
-            NCCL_TRY(n.Recv(pad, 4 * QPc, nt(), lf, g_comm.comm, s));
-        }
-        NCCL_TRY(n.GroupEnd());
-        NCCL_TRY(n.AllGather(interior(rb.Mpad[p->lg]), rb.Mfull[p->lg], 2 * nlg * QPc, nt(), g_comm.comm, s));
-        return FMMFFT_SUCCESS;
+        fmmfft_status_t st;
+        // NCCL work is issued in one order on every rank: the S halo (side stream) first
+        CUDA_TRY(cudaStreamWaitEvent(s, p->cs_done, 0));
+        if (p->L > p->lg && (st = exchange([this](const RankBufs& rb) { return sched_M(rb); }, s))) return st;
+        return allgather(s);
     }
 
     // M2L-B + REDUCE on the gathered base level (sources: all 2^B boxes, periodic)
@@ -1168,24 +1279,7 @@ struct Exec {
     // ---- the all-to-all: chunk r of W (k2 in r's block, own m) -> rank r's Rcv slot g
     fmmfft_status_t a2a() {
         if (p->G == 1) return FMMFFT_SUCCESS;
-        const int G = p->G;
-        const size_t chunk = (size_t)(p->P / G) * p->Mg;
-        if (p->virt) {
-            for (int r = 0; r < G; ++r)
-                for (int src = 0; src < G; ++src)
-                    CUDA_TRY(cudaMemcpyAsync((C*)p->ranks[r].Rcv + src * chunk, (C*)p->ranks[src].W + r * chunk,
-                                             chunk * sizeof(C), cudaMemcpyDeviceToDevice, s));
-            return FMMFFT_SUCCESS;
-        }
-        RankBufs& rb = p->ranks[0];
-        NcclApi& n = nccl();
-        NCCL_TRY(n.GroupStart());
-        for (int r = 0; r < G; ++r) {
-            NCCL_TRY(n.Send((C*)rb.W + r * chunk, 2 * chunk, nt(), r, g_comm.comm, s));
-            NCCL_TRY(n.Recv((C*)rb.Rcv + r * chunk, 2 * chunk, nt(), r, g_comm.comm, s));
-        }
-        NCCL_TRY(n.GroupEnd());
-        return FMMFFT_SUCCESS;
+        return exchange([this](const RankBufs& rb) { return sched_A2A(rb); }, s);
     }
 
     // one column pass of the four-step M-FFT (k_fft_col): nseq sequences of length 2^lMs
@@ -1311,6 +1405,26 @@ struct Exec {
         return FMMFFT_SUCCESS;
     }
 
+    // the k1 = 0 bins of the local M-FFT rows from the reductions r_p (k_dc_bins, reading R19)
+    fmmfft_status_t dc_bins() {
+        const int rows = p->P / p->G;
+        for (RankBufs& rb : p->ranks) {
+            // r_0: reduced by the per-level kernels (k_base*), or here from M^L's slot 0 when the
+            // fused per-FMM far field (p = 1..P-1 only) ran
+            const C* m0 = nullptr;
+            long long m0_n = 0, m0_stride = 0;
+            if (p->tree_p) {
+                m0 = interior(rb.Mpad[p->L]);
+                m0_n = (long long)p->nb * p->Q;
+                m0_stride = p->pmaj ? 1 : p->P;
+            }
+            launch_pdl(k_dc_bins<R>, (unsigned)((rows + 7) / 8), 256, 0, s, out[gidx(rb)], (const C*)rb.r, m0, m0_n,
+                       m0_stride, p->P, rows, grank(rb) * rows, (long long)p->M);
+            LAUNCH_CHECK();
+        }
+        return FMMFFT_SUCCESS;
+    }
+
     // inverse plans: y <- scale * conj(x) over this rank's N/G elements
     fmmfft_status_t conj_scale(const C* x, C* y, R scale) {
         const long long n = p->N / p->G;
@@ -1366,7 +1480,13 @@ struct Exec {
         fmmfft_status_t st;
         if (p->direct) return mfft();
 #define STEP(stage, call) if ((st = mark(stage))) return st; if ((st = call)) return st;
-        STEP(ST_COMM_S, comm_S())
+        if ((st = mark(ST_COMM_S))) return st;
+        if (p->G > 1) {                                 // S halo on the side stream (overlaps S2M)
+            CUDA_TRY(cudaEventRecord(p->fork, s));
+            CUDA_TRY(cudaStreamWaitEvent(side(), p->fork, 0));
+            if ((st = comm_S(side()))) return st;
+            CUDA_TRY(cudaEventRecord(p->cs_done, side()));
+        }
         STEP(ST_NEAR, near_up())
         STEP(ST_M2M, m2m_local())
         STEP(ST_COMM_M, comm_M())
@@ -1376,6 +1496,7 @@ struct Exec {
         STEP(ST_PFFT, post_pfft())
         STEP(ST_A2A, a2a())
         STEP(ST_MFFT, mfft())
+        if ((st = dc_bins())) return st;
 #undef STEP
         return mark(ST_COUNT);
     }
@@ -1545,6 +1666,7 @@ fmmfft_status_t fmmfft_comm_init(int rank, int G, const unsigned char id[128]) {
 
 fmmfft_status_t fmmfft_comm_destroy(void) {
     if (!g_comm.comm) return FMMFFT_SUCCESS;
+    if (g_comm_plans > 0) return fail(FMMFFT_INVALID_VALUE, "%d live plan(s) use the communicator: destroy them first", (int)g_comm_plans);
     NCCL_TRY(nccl().CommDestroy(g_comm.comm));
     g_comm = Comm{};
     return FMMFFT_SUCCESS;
@@ -1608,12 +1730,17 @@ static fmmfft_status_t plan_complex(fmmfft_plan_t* plan, long long N, int P, int
     if (B > 10) return fail(FMMFFT_UNSUPPORTED, "B > 10 not supported");
     if (nleaf % G) return fail(FMMFFT_INVALID_VALUE, "2^L %% G != 0");
     const bool virt = (flags & FMMFFT_FLAG_VIRTUAL) != 0;
-    if (G > 1 && !virt) {
+    const bool vnccl = (flags & FMMFFT_FLAG_VIRTUAL_NCCL) != 0;
+    if (vnccl && !virt) return fail(FMMFFT_INVALID_VALUE, "FMMFFT_FLAG_VIRTUAL_NCCL needs FMMFFT_FLAG_VIRTUAL");
+    if ((G > 1 && !virt) || vnccl) {
         if (!g_comm.comm) return fail(FMMFFT_NOT_INITIALIZED, "G > 1 needs fmmfft_comm_init");
-        if (g_comm.size != G) return fail(FMMFFT_INVALID_VALUE, "G=%d differs from the communicator size %d", G, g_comm.size);
+        const int want = vnccl ? 1 : G;
+        if (g_comm.size != want) return fail(FMMFFT_INVALID_VALUE, "communicator size %d, need %d", g_comm.size, want);
     }
     int dev = 0;
     CUDA_TRY(cudaGetDevice(&dev));
+    if (((G > 1 && !virt) || vnccl) && g_comm.device != dev)
+        return fail(FMMFFT_INVALID_VALUE, "current device %d differs from the communicator's device %d", dev, g_comm.device);
     cudaDeviceProp prop;
     CUDA_TRY(cudaGetDeviceProperties(&prop, dev));
     if (prop.major != 10 || prop.minor != 0)
@@ -1625,6 +1752,12 @@ static fmmfft_status_t plan_complex(fmmfft_plan_t* plan, long long N, int P, int
     p->N = N; p->P = P; p->G = G; p->B = B; p->Q = Q; p->M_L = M_L; p->L = L;
     p->inverse = (flags & FMMFFT_FLAG_INVERSE) != 0;
     p->M = N / P; p->Mg = p->M / G; p->prec = precision; p->flags = flags; p->virt = virt; p->device = dev;
+    if ((G > 1 && !virt) || vnccl) {
+        p->comm = g_comm.comm;
+        p->comm_rank = g_comm.rank;
+        p->vnccl = vnccl;
+        ++g_comm_plans;
+    }
     p->nb = (int)(nleaf / G);
     p->lg = std::min(std::max(B, ilog2(G) + 1), L);
     if (G == 1) p->lg = B;
@@ -1701,7 +1834,7 @@ static fmmfft_status_t plan_complex(fmmfft_plan_t* plan, long long N, int P, int
         const int nr = virt ? G : 1;
         p->ranks.resize(nr);
         for (int g = 0; g < nr && !st; ++g) {
-            p->ranks[g].g = virt ? g : (G > 1 ? g_comm.rank : 0);
+            p->ranks[g].g = virt ? g : p->comm_rank;
             st = alloc_rank(p, p->ranks[g]);
         }
     }
@@ -1721,6 +1854,7 @@ static fmmfft_status_t plan_complex(fmmfft_plan_t* plan, long long N, int P, int
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->fork, cudaEventDisableTiming);
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->join, cudaEventDisableTiming);
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->fork2, cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->cs_done, cudaEventDisableTiming);
         if (e == cudaSuccess && (flags & FMMFFT_FLAG_PROFILE)) {
             e = cudaEventCreate(&p->ev_s2t[0]);
             if (e == cudaSuccess) e = cudaEventCreate(&p->ev_s2t[1]);
@@ -1811,12 +1945,16 @@ fmmfft_status_t fmmfft_execute(fmmfft_plan_t p, const void* in, void* out, void*
     const char* b = (const char*)out;
     if (a < b + obytes && b < a + bytes) return fail(FMMFFT_INVALID_VALUE, "in and out overlap");
     if (((uintptr_t)in | (uintptr_t)out) & 15) return fail(FMMFFT_INVALID_VALUE, "in/out must be 16-byte aligned");
-    cudaPointerAttributes at;
+    cudaPointerAttributes at, bt;
     if (cudaPointerGetAttributes(&at, in) != cudaSuccess || at.type != cudaMemoryTypeDevice ||
-        cudaPointerGetAttributes(&at, out) != cudaSuccess || at.type != cudaMemoryTypeDevice) {
+        cudaPointerGetAttributes(&bt, out) != cudaSuccess || bt.type != cudaMemoryTypeDevice) {
         cudaGetLastError();
         return fail(FMMFFT_INVALID_VALUE, "in/out must be device pointers");
     }
+    if (at.device != p->device || bt.device != p->device)
+        return fail(FMMFFT_INVALID_VALUE, "in/out live on device %d/%d, the plan on device %d", at.device, bt.device, p->device);
+    DeviceGuard guard(p->device);
+    if (guard.err != cudaSuccess) return fail(FMMFFT_CUDA_ERROR, "cudaSetDevice(%d): %s", p->device, cudaGetErrorString(guard.err));
     cudaStream_t s = (cudaStream_t)stream;
     return p->prec == FMMFFT_C64 ? execute_t<float>(p, in, out, s) : execute_t<double>(p, in, out, s);
 }
@@ -1826,6 +1964,8 @@ fmmfft_status_t fmmfft_execute_host(fmmfft_plan_t p, const void* in_host, void* 
     const size_t nb = (size_t)(p->virt ? p->N : p->N / p->G) * p->esz;
     const size_t half = nb + (p->real ? p->esz : 0);        // real plans: N/2 + 1 complex values
     const size_t bytes = p->real && p->inverse ? half : nb, obytes = p->real && p->inverse ? nb : half;
+    DeviceGuard guard(p->device);
+    if (guard.err != cudaSuccess) return fail(FMMFFT_CUDA_ERROR, "cudaSetDevice(%d): %s", p->device, cudaGetErrorString(guard.err));
     RankBufs& rb = p->ranks[0];
     if (!rb.din) {
         fmmfft_status_t st;
@@ -1842,6 +1982,7 @@ fmmfft_status_t fmmfft_execute_host(fmmfft_plan_t p, const void* in_host, void* 
 
 fmmfft_status_t fmmfft_destroy(fmmfft_plan_t p) {
     if (!p) return FMMFFT_SUCCESS;
+    DeviceGuard guard(p->device);
     cudaDeviceSynchronize();
     destroy_plan(p);
     return FMMFFT_SUCCESS;
@@ -1865,7 +2006,10 @@ fmmfft_status_t fmmfft_stage_times(fmmfft_plan_t p, float* ms, int n, int* n_out
     CUDA_TRY(cudaEventSynchronize(p->ev[ST_COUNT]));
     const int k = std::min(n, (int)ST_COUNT + 1);
     for (int i = 0; i < k && i < ST_COUNT; ++i) CUDA_TRY(cudaEventElapsedTime(&ms[i], p->ev[i], p->ev[i + 1]));
-    if (k > ST_COUNT) CUDA_TRY(cudaEventElapsedTime(&ms[ST_COUNT], p->ev_s2t[0], p->ev_s2t[1]));
+    float s2t = 0.f;
+    if (!p->direct) CUDA_TRY(cudaEventElapsedTime(&s2t, p->ev_s2t[0], p->ev_s2t[1]));
+    if (k > ST_NEAR) ms[ST_NEAR] = std::max(0.f, ms[ST_NEAR] - s2t);     // S2T ran serialised inside it
+    if (k > ST_COUNT) ms[ST_COUNT] = s2t;
     *n_out = k;
     return FMMFFT_SUCCESS;
 }

@@ -155,8 +155,9 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
                         float* prh = &rh.x; float* prl = &rl.x; float* pih = &ihv.x; float* pil = &il.x;
 #pragma unroll
                         for (int q = 0; q < 4; ++q) {
-                            const float h1 = tc::to_tf32(re[q]); prh[q] = h1; prl[q] = re[q] - h1;
-                            const float h2 = tc::to_tf32(im[q]); pih[q] = h2; pil[q] = im[q] - h2;
+                            // lo rounded to nearest too (the MMA would truncate it: 2^-21 vs 2^-22)
+                            const float h1 = tc::to_tf32(re[q]); prh[q] = h1; prl[q] = tc::to_tf32(re[q] - h1);
+                            const float h2 = tc::to_tf32(im[q]); pih[q] = h2; pil[q] = tc::to_tf32(im[q] - h2);
                         }
                         const int off = k4 * S2TC_LBO_A + r * 16;   // [c][hi/lo][k4][row][16 B]
                         *reinterpret_cast<float4*>(As + 0 * S2TC_A_PART + off) = rh;

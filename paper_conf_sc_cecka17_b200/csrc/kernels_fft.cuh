@@ -722,20 +722,79 @@ k_fft_rowt(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, long long M, i
 // ---------------------------------------------------------------------------------------------
 template <typename R>
 __global__ void __launch_bounds__(256)
-k_conj_scale(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, long long n, R scale) {
+k_conj_scale(const C2<R>* in, C2<R>* out, long long n, R scale) {   // in == out allowed (no restrict / ldg)
     pdl_trigger();
     pdl_wait();
     const long long stride = (long long)gridDim.x * blockDim.x;
     for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; 2 * i < n; i += stride) {
         if constexpr (sizeof(R) == 4) {
-            const float4 v = __ldg(reinterpret_cast<const float4*>(in) + i);
+            const float4 v = reinterpret_cast<const float4*>(in)[i];
             reinterpret_cast<float4*>(out)[i] = make_float4(scale * v.x, -scale * v.y, scale * v.z, -scale * v.w);
         } else {
-            const double2 a = __ldg(in + 2 * i), b = __ldg(in + 2 * i + 1);
+            const double2 a = in[2 * i], b = in[2 * i + 1];
             out[2 * i] = make_double2(scale * a.x, -scale * a.y);
             out[2 * i + 1] = make_double2(scale * b.x, -scale * b.y);
         }
     }
+}
+
+// ---------------------------------------------------------------------------------------------
+// k_dc_bins: the k1 = 0 output of every local M-FFT row, y[M k2] = sum_p w_P^{p k2} r_p — eq. (1)
+// at k = M k2: sum_j x_j w_N^{j M k2} = sum_p w_P^{p k2} sum_m x_{p + P m} (reading R19). Through
+// the FMM these P bins are the sums of the far field over all M targets, a sum with heavy
+// cancellation (its terms ~ M / (pi d) against a net ~ M), so in float32 they carry ~1e-5 relative
+// error at M = 2^22 (growing like sqrt M) while every other bin is at ~1e-6; the reductions r_p of
+// Algorithm 1 line 11 hold the same quantities accurately. r_0 (p = 0 is no FMM) is
+// the sum of M^L's slot 0 (S2M columns sum to 1): read from r[0] when the level kernels reduced it,
+// else reduced here from M^L slot 0 (m0: m0_n values at stride m0_stride). Sums in float64.
+// ---------------------------------------------------------------------------------------------
+template <typename R>
+__global__ void __launch_bounds__(256)
+k_dc_bins(C2<R>* __restrict__ y, const C2<R>* __restrict__ r, const C2<R>* __restrict__ m0, long long m0_n,
+          long long m0_stride, int P, int rows, int row0, long long M) {
+    pdl_trigger();
+    __shared__ double2 red[8];
+    __shared__ double2 rr[1024];                                  // r_p (r_0 replaced), then summed
+    __shared__ double2 tw[1024];                                  // w_P^j, j < P
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    for (int j = tid; j < P; j += blockDim.x) tw[j] = twiddle_d(j, P);
+    pdl_wait();
+    for (int j = tid; j < P; j += blockDim.x) rr[j] = make_double2((double)r[j].x, (double)r[j].y);
+    if (m0 != nullptr) {                                          // r_0 = sum of M^L slot 0
+        double2 a = make_double2(0.0, 0.0);
+        for (long long i = tid; i < m0_n; i += blockDim.x) {
+            const C2<R> v = m0[i * m0_stride];
+            a.x += (double)v.x;
+            a.y += (double)v.y;
+        }
+        for (int o = 16; o > 0; o >>= 1) {                        // fixed-order reduction: deterministic
+            a.x += __shfl_xor_sync(0xffffffffu, a.x, o);
+            a.y += __shfl_xor_sync(0xffffffffu, a.y, o);
+        }
+        if (lane == 0) red[wid] = a;
+        __syncthreads();
+        if (tid == 0) {
+            double2 t = red[0];
+            for (int w = 1; w < (int)(blockDim.x >> 5); ++w) { t.x += red[w].x; t.y += red[w].y; }
+            rr[0] = t;
+        }
+    }
+    __syncthreads();
+    // one warp per output row: lanes over p, shuffle reduction
+    const int row = blockIdx.x * (blockDim.x >> 5) + wid;
+    if (row >= rows) return;
+    const int k2 = row0 + row;
+    double2 acc = make_double2(0.0, 0.0);
+    for (int pp = lane; pp < P; pp += 32) {
+        const double2 w = tw[(pp * k2) & (P - 1)], v = rr[pp];
+        acc.x += w.x * v.x - w.y * v.y;
+        acc.y += w.x * v.y + w.y * v.x;
+    }
+    for (int o = 16; o > 0; o >>= 1) {
+        acc.x += __shfl_xor_sync(0xffffffffu, acc.x, o);
+        acc.y += __shfl_xor_sync(0xffffffffu, acc.y, o);
+    }
+    if (lane == 0) y[(size_t)row * M] = C2<R>{(R)acc.x, (R)acc.y};
 }
 
 // ---------------------------------------------------------------------------------------------
@@ -788,8 +847,9 @@ k_c2r_pre(const C2<R>* __restrict__ X, C2<R>* __restrict__ Zc, long long H) {
     pdl_wait();
     const long long stride = (long long)gridDim.x * blockDim.x;
     for (long long k = (long long)blockIdx.x * blockDim.x + threadIdx.x; k <= H / 2; k += stride) {
-        const C2<R> a = X[k];
-        const C2<R> xb = X[H - k];
+        C2<R> a = X[k];
+        C2<R> xb = X[H - k];
+        if (k == 0) a.y = xb.y = R(0);     // X_0, X_H of a real signal are real: Im ignored (fmmfft.h)
         const R Er = R(0.5) * (a.x + xb.x), Ei = R(0.5) * (a.y - xb.y);   // (a + conj(xb)) / 2
         const R Dr = R(0.5) * (a.x - xb.x), Di = R(0.5) * (a.y + xb.y);   // (a - conj(xb)) / 2
         R wr, wi;                                                        // w_N^{-k} = exp(+2 pi i k / 2H)

@@ -15,7 +15,8 @@ import ctypes
 import torch
 
 from . import _lib
-from ._lib import C64, C128, FLAG_DEBUG, FLAG_DIRECT, FLAG_INVERSE, FLAG_PROFILE, FLAG_REAL, FLAG_VIRTUAL, check, lib
+from ._lib import (C64, C128, FLAG_DEBUG, FLAG_DIRECT, FLAG_INVERSE, FLAG_PROFILE, FLAG_REAL, FLAG_VIRTUAL,
+                   FLAG_VIRTUAL_NCCL, check, lib)
 
 _DT = {"c64": (C64, torch.complex64), "c128": (C128, torch.complex128)}
 
@@ -39,6 +40,14 @@ def init_comm(group=None) -> None:
         buf = buf.cuda()
     dist.broadcast(buf, src=0, group=group)
     check(lib.fmmfft_comm_init(rank, world, bytes(buf.cpu().numpy().tobytes())))
+
+
+def init_comm_local() -> None:
+    """A 1-rank NCCL communicator on the current device, no process group needed: the transport
+    of virtual plans created with transport="nccl" (FMMFFT_FLAG_VIRTUAL_NCCL)."""
+    raw = ctypes.create_string_buffer(128)
+    check(lib.fmmfft_get_unique_id(raw))
+    check(lib.fmmfft_comm_init(0, 1, raw.raw))
 
 
 def autotune(N: int, G: int = 1, precision: str = "c64", tol: float = 1e-5, measure: bool = True) -> dict:
@@ -68,17 +77,20 @@ class _DevView:
 class FmmFFT:
     def __init__(self, N: int, P: int, G: int = 1, B: int = 2, Q: int = 16, precision: str = "c64",
                  M_L: int = 64, virtual: bool = False, profile: bool = False, debug: bool = False,
-                 inverse: bool = False, direct: bool = False, real: bool = False):
+                 inverse: bool = False, direct: bool = False, real: bool = False, transport: str = "copy"):
         """direct=True: no FMM — the plain four-step FFT of length N on one GPU with the same M-FFT
         kernels (the in-house Cooley-Tukey comparator; P, B, Q, M_L ignored).
         real=True (FMMFFT_FLAG_REAL): N real inputs -> N/2+1 complex outputs; P, B, Q, M_L
-        describe the complex plan of length N/2 (G = 1)."""
+        describe the complex plan of length N/2 (G = 1).
+        transport="nccl" (virtual plans): the virtual ranks' exchanges through NCCL on a 1-rank
+        communicator (init_comm_local) instead of device copies."""
         self.N, self.P, self.G, self.B, self.Q, self.M_L = N, P, G, B, Q, M_L
         self.precision = precision
         self.virtual = virtual
         self._prec, self.dtype = _DT[precision]
         flags = (FLAG_VIRTUAL if virtual else 0) | (FLAG_PROFILE if profile else 0) | (FLAG_DEBUG if debug else 0) | \
-                (FLAG_INVERSE if inverse else 0) | (FLAG_DIRECT if direct else 0) | (FLAG_REAL if real else 0)
+                (FLAG_INVERSE if inverse else 0) | (FLAG_DIRECT if direct else 0) | (FLAG_REAL if real else 0) | \
+                (FLAG_VIRTUAL_NCCL if transport == "nccl" else 0)
         self.inverse = inverse
         self.real = real
         rdt = torch.float32 if precision == "c64" else torch.float64

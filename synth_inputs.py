@@ -45,16 +45,26 @@ def uniform_pm1(seed: int, counters: np.ndarray) -> np.ndarray:
 
 
 def complex_uniform(n0: int, count: int, seed: int = DEFAULT_SEED,
-                    dtype=np.complex128, chunk: int = 1 << 24) -> np.ndarray:
-    """x[n0 : n0+count] of the global seeded vector, as ``dtype`` (complex64 or complex128)."""
+                    dtype=np.complex128, chunk: int = 1 << 22) -> np.ndarray:
+    """x[n0 : n0+count] of the global seeded vector, as ``dtype`` (complex64 or complex128).
+    Chunks are filled by a thread pool (numpy releases the GIL); values depend only on n."""
     out = np.empty(count, dtype=dtype)
-    for a in range(0, count, chunk):
+
+    def fill(a):
         b = min(count, a + chunk)
         n = np.arange(n0 + a, n0 + b, dtype=np.uint64)
-        re = uniform_pm1(seed, np.uint64(2) * n)
-        im = uniform_pm1(seed, np.uint64(2) * n + np.uint64(1))
-        out[a:b].real = re
-        out[a:b].imag = im
+        out[a:b].real = uniform_pm1(seed, np.uint64(2) * n)
+        out[a:b].imag = uniform_pm1(seed, np.uint64(2) * n + np.uint64(1))
+
+    starts = range(0, count, chunk)
+    if count > 4 * chunk:
+        import os
+        from concurrent.futures import ThreadPoolExecutor
+        with ThreadPoolExecutor(max_workers=min(16, os.cpu_count() or 1)) as ex:
+            list(ex.map(fill, starts))
+    else:
+        for a in starts:
+            fill(a)
     return out
 
 

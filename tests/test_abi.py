@@ -105,7 +105,8 @@ def test_flag_values_match_header(L):
     src = open(os.path.join(ROOT, "include", "fmmfft.h")).read()
     hdr = {m[0]: int(m[1]) for m in re.findall(r"#define FMMFFT_FLAG_(\w+)\s+(\d+)u", src)}
     assert hdr == {"VIRTUAL": L.FLAG_VIRTUAL, "PROFILE": L.FLAG_PROFILE, "DEBUG": L.FLAG_DEBUG,
-                   "INVERSE": L.FLAG_INVERSE, "DIRECT": L.FLAG_DIRECT, "REAL": L.FLAG_REAL}
+                   "INVERSE": L.FLAG_INVERSE, "DIRECT": L.FLAG_DIRECT, "REAL": L.FLAG_REAL,
+                   "VIRTUAL_NCCL": L.FLAG_VIRTUAL_NCCL}
 
 
 def test_real_multi_gpu_unsupported(L):

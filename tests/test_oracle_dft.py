@@ -171,3 +171,23 @@ def test_rdft_cosine(N, k0):
     expect = np.zeros(N // 2 + 1, dtype=complex)
     expect[k0] = N / 2
     assert np.max(np.abs(y - expect)) < 1e-10 * N
+
+
+@pytest.mark.parametrize("N,J", [(1024, 32), (4096, 64), (4096, 4096), (2048, 1)])
+def test_dft_at_matches_direct_and_radix2(N, J):
+    # dft_at is eq. (1) evaluated at selected k with the exponent split j = j1 + J j2: it must
+    # reproduce the brute-force sum and the radix-2 FFT at every k
+    x = SI.complex_uniform(0, N, seed=7)
+    ks = np.arange(N)
+    y = O.dft_at(x, ks, J=J)
+    scale = np.sqrt(N)
+    assert np.max(np.abs(y - O.dft_direct(x))) < 1e-13 * scale * 10
+    assert np.max(np.abs(y - O.fft_radix2(x))) < 1e-13 * scale * 10
+
+
+def test_dft_at_closed_forms():
+    N = 1 << 16
+    k = np.array([0, 1, 4321, N - 1])
+    assert np.max(np.abs(O.dft_at(SI.delta(N, 777), k) - np.exp(-2j * np.pi * ((777 * k) % N) / N))) < 1e-12
+    y = O.dft_at(SI.tone(N, 4321), k)
+    assert abs(y[2] - N) < 1e-8 * N and np.max(np.abs(y[[0, 1, 3]])) < 1e-8 * N
