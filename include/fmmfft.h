@@ -188,7 +188,6 @@ typedef struct {
 #define FMMFFT_VARIANT_S2T_TC     2u  /* near field on tcgen05 tensor cores (3xTF32)             */
 #define FMMFFT_VARIANT_ROW_FFT1   4u  /* M-point FFTs as one single-pass kernel per row        */
 #define FMMFFT_VARIANT_FOURSTEP   8u  /* long rows: column pass(es) + transposing row pass     */
-#define FMMFFT_VARIANT_ROW_CL    16u  /* rows split over a cluster of CTAs (k_fft_rowc)        */
 #define FMMFFT_VARIANT_DOWN_LVL  32u  /* wide levels on the per-level M2M / M2L kernels        */
 #define FMMFFT_VARIANT_PMAJ      64u  /* leaf M^L / L^L stored p-major [p][b][q] (the cluster far
                                          field; never with FMMFFT_FLAG_DEBUG): the debug buffers of

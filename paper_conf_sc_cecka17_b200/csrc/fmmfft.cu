@@ -11,7 +11,7 @@
 //   comm_M    M^l halos for l > l_g (line 7) + all-gather of level l_g (line 9, reading R16)
 //   top       M2M l_g-1 .. B on the gathered level, M2L-B (line 10) + REDUCE (line 11),
 //             M2L + L2L for B < l <= l_g (replicated top of the tree)
-//   down      M2L-l (line 8) + L2L (line 13) for l = l_g+1 .. L   k_down per level
+//   down      M2L-l (line 8) + L2L (line 13) for l = l_g+1 .. L   k_tree_down + k_m2l_lvl
 //   post_pfft L2T + POST + P-point FFTs + transposed store (lines 14-16)
 //   a2a       the one all-to-all transpose (line 16)
 //   mfft      P/G M-point FFTs, multi-pass Stockham (line 16)
@@ -235,21 +235,14 @@ struct fmmfft_plan_s {
     std::vector<void*> m2l_pmaj;     // p-major copies for the fused per-p tree (G = 1), by level
     bool tree_p = false;             // use k_tree_p for the far field
     int tree_cl = 1;                 // k_tree_pc: CTAs per FMM (cluster), 1 = not used
-    bool tree_phased = false;        // ... as up / all-levels M2L / L2L-chain launches (FMMFFT_TREE=p) (k_tree_pq<.., false>, k_m2l_flat, k_tree_dn)
     int fs_lc1 = 0, fs_lc2 = 0, fs_lr = 0;   // four-step large-M FFT: column pass bits (2nd: 0 = none), row pass bits
-    int s2m_nbx = 0, s2m_pc = 0, pp_ms = 0;  // tuning knobs (FMMFFT_S2M_NBX, FMMFFT_S2M_PC, FMMFFT_PP_MS); 0 = default
     bool inverse = false;            // FMMFFT_FLAG_INVERSE: x = F_N^{-1} y
     bool real = false;               // FMMFFT_FLAG_REAL: N (below) is the complex length H = N_real / 2
-    bool pp_old = false;             // FMMFFT_PP=tile: the shared-memory-tile k_post_pfft for every P
-    bool fs_narrow = false;          // FMMFFT_FS_NARROW=1: 11-bit (c64) / 10-bit (c128) four-step passes on 4-column CTAs
     bool pmaj = false;               // M^L / L^L p-major [p][b][q] between k_s2m, k_tree_pc and post_pfft
-    int s2t_tpc = 0;                 // FMMFFT_S2T_TPC: tiles per k_s2t_tc CTA (0 = one wave)
     bool direct = false;             // FMMFFT_FLAG_DIRECT: plain four-step FFT of length N, no FMM
-    bool lvl_off = false;            // FMMFFT_DOWN=tree: every down level in k_tree_down (no k_m2l_lvl)
     bool s2t_tc = false;             // S2T on tcgen05 (k_s2t_tc): complex64, M_L = 64, nb % 128 == 0
     void* toep = nullptr;            // its Toeplitz hi/lo operand table
     bool row_fft1 = false;           // M-point FFTs in one pass per row (k_fft_row), M fits smem
-    int row_cl = 0;                  // ... on a cluster of row_cl CTAs per row (k_fft_rowc), 0 = off
     void* twM = nullptr;             // its twiddles w_M^u, u < M/16
     std::vector<fmmfft::RankBufs> ranks;
     std::vector<int> radices;        // M-FFT passes
@@ -407,7 +400,7 @@ static fmmfft_status_t build_tables(fmmfft_plan_s* p) {
         rho[2 * pp + 1] = pp ? -std::sin(M_PI * pp / P) * sn : 0.0;
     }
     if ((st = upload<R>(p, &p->rho, rho))) return st;
-    if (p->row_fft1 || p->row_cl) {                      // w_M^u = exp(-2 pi i u / M), u < M/16
+    if (p->row_fft1) {                                   // w_M^u = exp(-2 pi i u / M), u < M/16
         std::vector<double> tw(2 * (p->M / 16));
         for (long long u = 0; u < p->M / 16; ++u) {
             tw[2 * u] = std::cos(2 * M_PI * (double)u / (double)p->M);
@@ -451,6 +444,22 @@ static void choose_fourstep(fmmfft_plan_s* p, int lM, int mx) {
         p->fs_lc2 = lM - p->fs_lr - p->fs_lc1;
     }
     if (p->fs_lc1 < 5 || p->fs_lr < 5 || (p->fs_lc2 && p->fs_lc2 < 5)) p->fs_lr = p->fs_lc1 = p->fs_lc2 = 0;
+}
+
+// the M-point row FFT kernels for p->M, p->P / p->G rows: one pass per row in shared memory
+// (k_fft_row, M <= 2^14 / 2^13) when there are enough rows to fill the GPU, else the four-step
+// column + transposing row passes, else the multi-pass Stockham kernel (short rows).
+// FMMFFT_MFFT=pass forces k_fft_pass, =fs the four-step (test knobs).
+static void plan_mfft(fmmfft_plan_s* p) {
+    plan_radices(p);
+    const int lM = ilog2(p->M);
+    const char* e = getenv("FMMFFT_MFFT");
+    const bool pass = e && e[0] == 'p', fs = e && e[0] == 'f';
+    p->row_fft1 = !pass && lM >= 8 && lM <= (p->prec == FMMFFT_C64 ? 14 : 13);
+    const bool few_rows = p->P / p->G < 148 && lM >= 13;
+    if ((fs && lM >= 10) || few_rows) p->row_fft1 = false;
+    // 11-bit passes (1 CTA per SM) measured slower than 3 passes of <= 10 bits
+    if (!pass && !p->row_fft1) choose_fourstep(p, lM, 10);
 }
 
 static fmmfft_status_t alloc_rank(fmmfft_plan_s* p, RankBufs& rb) {
@@ -537,7 +546,6 @@ static fmmfft_status_t init_kernel_attrs() {
                 dispatch<4, 5, 6, 7>(lml, [&](auto v) { set((const void*)k_s2m<R, PCv, decltype(v)::value>); });
             if constexpr (PCv <= (sizeof(R) == 4 ? 16 : 8)) {
                 set((const void*)k_up<R, PCv>);
-                set((const void*)k_m2l_flat<R, 8, PCv>);
                 set((const void*)k_base<R, 4, PCv>);
                 set((const void*)k_base<R, 8, PCv>);
                 set((const void*)k_base<R, 16, PCv>);
@@ -551,16 +559,8 @@ static fmmfft_status_t init_kernel_attrs() {
         };
         for (int pc = 2; pc <= (sizeof(R) == 4 ? 32 : 16); pc *= 2) dispatch<2, 4, 8, 16, 32>(pc, per_pc);
         if constexpr (sizeof(R) == 4) {
-            set((const void*)k_tree_pq<16, 512, 8>);
-            set((const void*)k_tree_pq<16, 512, 8, false>);
-            set((const void*)k_tree_pq<8, 512, 8, false>);
-            set((const void*)k_tree_dn<16, 512>);
-            set((const void*)k_tree_dn<8, 512>);
-            set((const void*)k_tree_pq<8, 512, 8>);
             set((const void*)k_tree_pc<16, 512, 2>);
-            set((const void*)k_tree_pc<16, 256, 4>);
             set((const void*)k_tree_pc<8, 512, 2>);
-            set((const void*)k_tree_pc<8, 256, 4>);
         }
         if constexpr (sizeof(R) == 4) { set((const void*)k_s2t_tc<1>); set((const void*)k_s2t_tc<2>); }
         set((const void*)k_base_sg<R, 4, sizeof(R) == 4 ? 8 : 4, 4>);
@@ -589,24 +589,12 @@ static fmmfft_status_t init_kernel_attrs() {
             });
         for (int lr = 1; lr <= 10; ++lr)
             dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10>(lr, [&](auto v) { set((const void*)k_fft_pass<R, decltype(v)::value>); });
-        for (int lk = 8; lk <= kRowFftMax<R> - 1; ++lk)
-            dispatch<8, 9, 10, 11, 12, 13>(lk, [&](auto v) {
-                constexpr int LK = decltype(v)::value;
-                if constexpr (LK <= kRowFftMax<R> - 1) {
-                    set((const void*)k_fft_rowc<R, LK, 2>);
-                    set((const void*)k_fft_rowc<R, LK, 4>);
-                }
-            });
         for (int l = 5; l <= fs_max<R>(); ++l)
             dispatch<5, 6, 7, 8, 9, 10, 11>(l, [&](auto v) {
                 constexpr int LV = decltype(v)::value;
                 if constexpr (LV <= fs_max<R>()) {
                     set((const void*)k_fft_col<R, LV, fs_cols<R>(LV)>);
                     set((const void*)k_fft_rowt<R, LV, fs_cols<R>(LV)>);
-                    if constexpr (LV >= fs_max<R>() - 1) {
-                        set((const void*)k_fft_col<R, LV, 4>);
-                        set((const void*)k_fft_rowt<R, LV, 4>);
-                    }
                 }
             });
         for (int ll = 8; ll <= kRowFftMax<R>; ++ll)
@@ -812,12 +800,12 @@ struct Exec {
     // post_pfft), so the far field and the near field run concurrently
     fmmfft_status_t near_up() {
         fmmfft_status_t st;
-        const int PCs = std::min(p->P, p->s2m_pc ? p->s2m_pc : (sizeof(R) == 4 ? 32 : 16));
+        const int PCs = std::min(p->P, sizeof(R) == 4 ? 32 : 16);
         for (RankBufs& rb : p->ranks) {
             const C* S = in[p->virt ? rb.g : 0];
             const int Qp = (p->Q + 3) / 4 * 4;
             // boxes per CTA (k_s2m NBX <= 2; nb is even or 1): 1 unless that gives > 4 CTAs per SM
-            int nbx = p->s2m_nbx ? p->s2m_nbx : ((long long)p->nb * (p->P / PCs) > 4 * 148 ? 2 : 1);
+            int nbx = (long long)p->nb * (p->P / PCs) > 4 * 148 ? 2 : 1;
             if (p->nb < 2) nbx = 1;
             const size_t smem = (size_t)2 * p->M_L * (PCs + 1) * sizeof(C) + (size_t)Qp * p->M_L * sizeof(R);
             const dim3 grid((unsigned)(p->nb / nbx), (unsigned)(p->P / PCs));
@@ -843,7 +831,6 @@ struct Exec {
                 // (one CTA per SM: TMEM + ~180 KB of shared memory)
                 const int cpp = std::max(1, 148 / (p->P - 1));             // CTAs per p
                 int tpc = (ntile + cpp - 1) / cpp;
-                if (p->s2t_tpc) tpc = std::min(ntile, p->s2t_tpc);
                 for (RankBufs& rb : p->ranks) {
                     const dim3 grid((unsigned)((ntile + tpc - 1) / tpc), (unsigned)(p->P - 1));
                     // several tiles per CTA: A chunks prefetched two ahead; one tile: one ahead (the
@@ -906,7 +893,7 @@ struct Exec {
         long long nbc = nb_from;
         // wide levels: one register-blocked k_m2m_lvl launch per level (>= 2 tiles of parents)
         constexpr int PCl = lvl_pc<R>();
-        const bool lvl_ok = !p->lvl_off && (p->Q == 8 || p->Q == 16 || p->Q == 24) && p->PCd % PCl == 0 && p->P % PCl == 0;
+        const bool lvl_ok = (p->Q == 8 || p->Q == 16 || p->Q == 24) && p->PCd % PCl == 0 && p->P % PCl == 0;
         int optin = 0;
         CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, p->device));
         while (lvl_ok && cur > to && (nbc >> 1) >= 2 * lvl_nt<R, 16>() &&
@@ -961,65 +948,13 @@ struct Exec {
             a.dbg = (p->flags & FMMFFT_FLAG_DEBUG) ? 1 : 0;
             a.pmaj = p->pmaj ? 1 : 0;
             const int tabB = ((1 << p->B) - 3) * p->Q * p->Q;
-            // complex64 with Q = 16 or 8 and <= 8 boxes per thread group: register-blocked kernel
+            // complex64, Q = 16 or 8: each FMM on a cluster of 2 CTAs (k_tree_pc)
             if constexpr (sizeof(R) == 4) {
-                const int ngrp = 512 / p->Q;
-                if ((p->Q == 16 || p->Q == 8) && (1LL << p->L) <= 8LL * ngrp && p->tree_phased) {
-                    // (1) M2M + M2L-B + REDUCE per FMM, (2) all levels' M2L in one wide launch,
-                    // (3) the L2L chain per FMM
-                    const size_t smem1 = tree_p_smem(p, 512);
-                    if (p->Q == 16) launch_pdl(k_tree_pq<16, 512, 8, false>, p->P - 1, 512, smem1, s, a, (const float*)p->m2m, p->P, tabB);
-                    else            launch_pdl(k_tree_pq<8, 512, 8, false>, p->P - 1, 512, smem1, s, a, (const float*)p->m2m, p->P, tabB);
-                    LAUNCH_CHECK();
-                    if (p->L > p->B) {
-                        M2LFlat f{};
-                        constexpr int BR = 8;
-                        int tiles = 0;
-                        for (int lev = p->B + 1; lev <= p->L; ++lev) {
-                            f.src[lev] = interior(rb.Mpad[lev]);
-                            f.out[lev] = rb.Lloc[lev];
-                            f.tab[lev] = p->m2l[lev];
-                            f.tile0[lev] = tiles;
-                            tiles += ((1 << lev) + BR - 1) / BR;
-                        }
-                        f.tile0[p->L + 1] = tiles;
-                        f.lmin = p->B + 1;
-                        f.lmax = p->L;
-                        const int PC_ = p->PCd;
-                        const size_t smem2 = (size_t)(BR + 4 + BR / 2) * p->Q * PC_ * sizeof(C) + (size_t)p->m2l_chunk * sizeof(R) +
-                                             (size_t)2 * p->Q * p->Q * sizeof(R) + (BR + 4) * sizeof(int);
-                        const dim3 grid((unsigned)tiles, (unsigned)(p->P / PC_));
-                        with_pcd([&](auto pc) {
-                            constexpr int PCv = decltype(pc)::value;
-                            launch_pdl(k_m2l_flat<R, BR, PCv>, grid, PCv * p->Q, smem2, s, f, p->m2l_chunk, (const R*)p->m2m, p->P, p->Q);
-                        });
-                        LAUNCH_CHECK();
-                        const size_t smem3 = (((size_t)2 << p->L) - ((size_t)1 << p->B)) * p->Q * sizeof(C) + (size_t)2 * p->Q * p->Q * sizeof(R);
-                        if (p->Q == 16) launch_pdl(k_tree_dn<16, 512>, p->P - 1, 512, smem3, s, a, (const float*)p->m2m, p->P);
-                        else            launch_pdl(k_tree_dn<8, 512>, p->P - 1, 512, smem3, s, a, (const float*)p->m2m, p->P);
-                        LAUNCH_CHECK();
-                    }
-                    continue;
-                }
-                if (p->tree_cl > 1) {                            // cluster of CL CTAs per FMM (k_tree_pc)
-                    const size_t smem = tree_pc_smem(p, p->tree_cl);
-                    const unsigned grid = (unsigned)((p->P - 1) * p->tree_cl);
-                    if (p->tree_cl == 2) {
-                        if (p->Q == 16) launch_cluster(k_tree_pc<16, 512, 2>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
-                        else            launch_cluster(k_tree_pc<8, 512, 2>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
-                    } else {
-                        if (p->Q == 16) launch_cluster(k_tree_pc<16, 256, 4>, grid, 256, smem, s, a, (const float*)p->m2m, p->P, tabB);
-                        else            launch_cluster(k_tree_pc<8, 256, 4>, grid, 256, smem, s, a, (const float*)p->m2m, p->P, tabB);
-                    }
-                    LAUNCH_CHECK();
-                    continue;
-                }
-                if ((p->Q == 16 || p->Q == 8) && (1LL << p->L) <= 8LL * ngrp) {
-                    // + L2L rows as float2 + the two alternating L^l buffers (2^L and 2^(L-1) boxes)
-                    const size_t smem = tree_p_smem(p, 512) + (size_t)p->Q * p->Q * 2 * sizeof(R) +
-                                        (((size_t)3 * p->Q) << (p->L - 1)) * sizeof(C);
-                    if (p->Q == 16) launch_plain(k_tree_pq<16, 512, 8>, p->P - 1, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
-                    else            launch_plain(k_tree_pq<8, 512, 8>, p->P - 1, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
+                if (p->tree_cl == 2) {
+                    const size_t smem = tree_pc_smem(p, 2);
+                    const unsigned grid = (unsigned)((p->P - 1) * 2);
+                    if (p->Q == 16) launch_cluster(k_tree_pc<16, 512, 2>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
+                    else            launch_cluster(k_tree_pc<8, 512, 2>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
                     LAUNCH_CHECK();
                     continue;
                 }
@@ -1141,7 +1076,6 @@ struct Exec {
     // first level handled by the per-level kernel k_m2l_lvl (levels with >= 2 tiles per rank);
     // the levels above it go to k_tree_down. FMMFFT_DOWN=tree keeps every level in k_tree_down.
     int lvl_first() const {
-        if (p->lvl_off) return p->L + 1;
         if (!(p->Q == 8 || p->Q == 16 || p->Q == 24)) return p->L + 1;
         constexpr int PCl = lvl_pc<R>();
         if (p->PCd % PCl || p->P % PCl) return p->L + 1;
@@ -1232,7 +1166,7 @@ struct Exec {
     // ---- L2T + POST + P-FFT
     fmmfft_status_t post_pfft() {
         // P <= 32 (and a specialised Q): the register-resident variant, one thread per (box, m)
-        if (p->P <= 32 && p->P >= 2 && (p->Q == 8 || p->Q == 16 || p->Q == 24) && p->M_L <= 256 && !p->pp_old) {
+        if (p->P <= 32 && p->P >= 2 && (p->Q == 8 || p->Q == 16 || p->Q == 24) && p->M_L <= 256) {
             const int nbx = std::max(1, std::min(p->nb, 256 / p->M_L));
             if (p->nb % nbx == 0) {
                 const size_t smem = ((size_t)nbx * p->Q * p->P + 2 * p->P + 16) * sizeof(C);
@@ -1255,7 +1189,6 @@ struct Exec {
         // leaves fewer than ~4 CTAs per SM (small N: latency-bound, more CTAs in flight)
         int MS = std::min(p->M_L, std::max(1, TILE / p->P));
         while (MS > 16 && (long long)p->nb * (p->M_L / MS) < 4 * 148) MS /= 2;
-        if (p->pp_ms) MS = std::min(p->M_L, p->pp_ms);
         const int threads = std::min(sizeof(R) == 4 ? 1024 : 512, std::max(32, MS * p->P / 8));
         size_t smem = (size_t)MS * (p->P + 1) * sizeof(C) + (size_t)p->P * sizeof(C) + (size_t)p->Q * MS * sizeof(R);
         const int stage_L = smem + (size_t)(p->Q + 1) * p->P * sizeof(C) <= 160 * 1024;   // stage L^L of the box
@@ -1283,20 +1216,14 @@ struct Exec {
     }
 
     // one column pass of the four-step M-FFT (k_fft_col): nseq sequences of length 2^lMs
+    // (lMi_ >= 0: inner count given explicitly, then lMs only sets the twiddle w_{2^lMs}; 0 = none)
     fmmfft_status_t col_pass(const C* in_, C* out_, int LCv, int lMs, int lSdiv, long long in_row, int lblk,
-                             long long blk_stride, long long nseq) {
-        const int lMi = lMs - LCv;
+                             long long blk_stride, long long nseq, int lMi_ = -1) {
+        const int lMi = lMi_ >= 0 ? lMi_ : lMs - LCv;
         bool ok = dispatch<5, 6, 7, 8, 9, 10, 11>(LCv, [&](auto lc) {
             constexpr int LC = decltype(lc)::value;
             constexpr int CB = fs_cols<R>(LC);
             if constexpr (LC <= fs_max<R>()) {
-                if constexpr (LC >= fs_max<R>() - 1) {
-                    if (p->fs_narrow) {             // 4 columns (32-byte runs): ~70 KB, several CTAs per SM
-                        launch_pdl(k_fft_col<R, LC, 4>, dim3((unsigned)((1LL << lMi) / 4), (unsigned)nseq), 4 << (LC - 4),
-                                   fft_col_smem<R, LC, 4>(), s, in_, out_, lMs, lMi, lSdiv, (long long)p->M, in_row, lblk, blk_stride);
-                        return;
-                    }
-                }
                 launch_pdl(k_fft_col<R, LC, CB>, dim3((unsigned)((1LL << lMi) / CB), (unsigned)nseq), CB << (LC - 4),
                            fft_col_smem<R, LC, CB>(), s, in_, out_, lMs, lMi, lSdiv, (long long)p->M, in_row, lblk, blk_stride);
             }
@@ -1306,19 +1233,22 @@ struct Exec {
         return FMMFFT_SUCCESS;
     }
 
-    // ---- M-point FFTs over the P/G local rows
-    fmmfft_status_t mfft() {
+    // ---- M-point FFTs over the P/G local rows (line 16): from the all-to-all receive
+    // layout (G > 1: [src][row][m_local(src)]) or the P-FFT output [row][m] (G = 1), into `dst`
+    // (default: the caller's output) in natural order
+    fmmfft_status_t mfft(const C* src_override = nullptr, bool to_tn = false) {
         fmmfft_status_t st_;
         const int n = (int)p->radices.size();
         const long long rows = p->P / p->G;
         const int lM = ilog2(p->M);
         for (RankBufs& rb : p->ranks) {
-            C* dst = out[p->virt ? rb.g : 0];
-            const C* src = p->direct ? in[0] : (const C*)(p->G > 1 ? rb.Rcv : rb.W);
+            C* dst = to_tn ? (C*)rb.Tn : out[gidx(rb)];
+            const C* src = src_override ? src_override : (const C*)(p->G > 1 ? rb.Rcv : rb.W);
+            if (src_override == in[0] && p->virt) src = in[gidx(rb)];
+            long long in_row = p->M, blk_stride = 0;
+            int lblk = 62;
+            if (p->G > 1 && src_override != in[0]) { in_row = p->Mg; lblk = ilog2(p->Mg); blk_stride = (p->P / p->G) * p->Mg; }
             if (p->fs_lr) {                      // four-step: column pass(es) + transposing row pass
-                long long in_row = p->M, blk_stride = 0;
-                int lblk = 62;
-                if (p->G > 1) { in_row = p->Mg; lblk = ilog2(p->Mg); blk_stride = (p->P / p->G) * p->Mg; }
                 const int npass = p->fs_lc2 ? 3 : 2;
                 C* a1out = npass == 3 ? dst : (C*)rb.tmp;
                 if ((st_ = col_pass(src, a1out, p->fs_lc1, lM, 0, in_row, lblk, blk_stride, rows))) return st_;
@@ -1333,47 +1263,21 @@ struct Exec {
                 bool ok = dispatch<5, 6, 7, 8, 9, 10, 11>(p->fs_lr, [&](auto ll) {
                     constexpr int LL = decltype(ll)::value;
                     constexpr int CR = fs_cols<R>(LL);
-                    if constexpr (LL <= fs_max<R>()) {
-                        if constexpr (LL >= fs_max<R>() - 1) {
-                            if (p->fs_narrow) {
-                                launch_pdl(k_fft_rowt<R, LL, 4>, (unsigned)(trows / 4), 4 << (LL - 4), fft_rowt_smem<R, LL, 4>(), s,
-                                           bsrc, dst, (long long)p->M, lrpr);
-                                return;
-                            }
-                        }
+                    if constexpr (LL <= fs_max<R>())
                         launch_pdl(k_fft_rowt<R, LL, CR>, (unsigned)(trows / CR), CR << (LL - 4), fft_rowt_smem<R, LL, CR>(), s,
                                    bsrc, dst, (long long)p->M, lrpr);
-                    }
                 });
                 if (!ok) return fail(FMMFFT_UNSUPPORTED, "k_fft_rowt: 2^%d", p->fs_lr);
                 LAUNCH_CHECK();
                 continue;
             }
-            if (p->row_cl) {                     // one pass per row on a cluster of row_cl CTAs
-                int in_row = (int)p->M, lblk = lM, blk_stride = 0;
-                if (p->G > 1) { in_row = (int)p->Mg; lblk = ilog2(p->Mg); blk_stride = (int)((p->P / p->G) * p->Mg); }
-                const int LKr = lM - ilog2(p->row_cl);
-                const size_t smem = ((size_t)(1 << LKr) + (1 << LKr) / 16 + p->M / 16 + 16 * p->row_cl) * sizeof(C);
-                const unsigned grid = (unsigned)(rows * p->row_cl);
-                dispatch<8, 9, 10, 11, 12, 13>(LKr, [&](auto lk) {
-                    constexpr int LK = decltype(lk)::value;
-                    if constexpr (LK <= kRowFftMax<R> - 1) {
-                        if (p->row_cl == 2) launch_cluster(k_fft_rowc<R, LK, 2>, grid, 1 << (LK - 4), smem, s, src, dst, (const C*)p->twM, in_row, lblk, blk_stride);
-                        else                launch_cluster(k_fft_rowc<R, LK, 4>, grid, 1 << (LK - 4), smem, s, src, dst, (const C*)p->twM, in_row, lblk, blk_stride);
-                    }
-                });
-                LAUNCH_CHECK();
-                continue;
-            }
             if (p->row_fft1) {                   // one pass per row, the row in shared memory
-                int in_row = (int)p->M, lblk = lM, blk_stride = 0;
-                if (p->G > 1) { in_row = (int)p->Mg; lblk = ilog2(p->Mg); blk_stride = (int)((p->P / p->G) * p->Mg); }
                 const size_t smem = ((size_t)p->M + p->M / 16 + p->M / 16) * sizeof(C);
                 dispatch<8, 9, 10, 11, 12, 13, 14>(lM, [&](auto ll) {
                     constexpr int LL = decltype(ll)::value;
                     if constexpr (LL <= kRowFftMax<R>)
                         launch_pdl(k_fft_row<R, LL>, (unsigned)rows, 1 << (LL - 4), smem, s, src, dst, (const C*)p->twM,
-                                   in_row, lblk, blk_stride);
+                                   (int)in_row, lblk == 62 ? lM : lblk, (int)blk_stride);
                 });
                 LAUNCH_CHECK();
                 continue;
@@ -1385,9 +1289,9 @@ struct Exec {
                 const long long nj = p->M / Rp;
                 long long c = std::min<long long>(TILE / Rp, nj);
                 while (c > 8 && c * Rp > 2048 && (nj / c) * rows < 2 * 148) c /= 2;
-                int in_row = (int)p->M, lblk = lM, blk_stride = 0;
-                if (i == 0 && p->G > 1) {
-                    in_row = (int)p->Mg; lblk = ilog2(p->Mg); blk_stride = (int)((p->P / p->G) * p->Mg);
+                int ir = (int)p->M, lb = lM, bs = 0;
+                if (i == 0 && blk_stride) {
+                    ir = (int)in_row; lb = lblk; bs = (int)blk_stride;
                     c = std::min<long long>(c, p->Mg);
                 }
                 const int threads = (int)std::min<long long>(sizeof(R) == 4 ? 1024 : 512, std::max<long long>(32, c * Rp / 8));
@@ -1395,7 +1299,7 @@ struct Exec {
                 const dim3 grid((unsigned)(nj / c), (unsigned)rows);
                 dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10>(lR, [&](auto lr) {
                     constexpr int LR = decltype(lr)::value;
-                    launch_pdl(k_fft_pass<R, LR>, grid, threads, smem, s, src, o, lM, lNs, ilog2(c), in_row, lblk, blk_stride);
+                    launch_pdl(k_fft_pass<R, LR>, grid, threads, smem, s, src, o, lM, lNs, ilog2(c), ir, lb, bs);
                 });
                 LAUNCH_CHECK();
                 src = o;
@@ -1476,9 +1380,40 @@ struct Exec {
         return FMMFFT_SUCCESS;
     }
 
+    // ---- the distributed radix-P Cooley-Tukey FFT with three all-to-alls (FMMFFT_FLAG_DIRECT,
+    // G > 1): the same exchange schedule, M-FFT kernels and column
+    // pass as the FMM-FFT, so the two differ only in the FMM vs the two extra transposes
+    fmmfft_status_t run_direct_dist() {
+        fmmfft_status_t st;
+        const long long Mg = p->Mg, rows = p->P / p->G;
+        auto a2a_ = [this]() { return exchange([this](const RankBufs& rb) { return sched_A2A(rb); }, s); };
+        for (RankBufs& rb : p->ranks) {                 // (1) [m_local][p] -> [p][m_local]
+            const dim3 grid((unsigned)((p->P + 31) / 32), (unsigned)((Mg + 31) / 32));
+            launch_pdl(k_transpose_rc<R>, grid, dim3(32, 8), 0, s, in[gidx(rb)], (C*)rb.W, Mg, (long long)p->P);
+            LAUNCH_CHECK();
+        }
+        if ((st = a2a_())) return st;                   //     transpose P-major -> M-major
+        if ((st = mfft(nullptr, true))) return st;      // (2) P/G local M-point FFTs -> Tn
+        for (RankBufs& rb : p->ranks) {                 // (3) twiddle + (4)'s send layout
+            const unsigned blocks = (unsigned)std::min<long long>((p->M * rows + 255) / 256, 148LL * 8);
+            launch_pdl(k_twiddle_chunk<R>, blocks, 256, 0, s, (const C*)rb.Tn, (C*)rb.W, (long long)p->M, ilog2(Mg),
+                       ilog2(rows), (long long)grank(rb) * rows, p->N);
+            LAUNCH_CHECK();
+        }
+        if ((st = a2a_())) return st;                   //     transpose M-major -> P-major
+        for (RankBufs& rb : p->ranks)                   // (5) M/G local P-point FFTs (columns of [p][k1_local])
+            if ((st = col_pass((const C*)rb.Rcv, (C*)rb.W, ilog2(p->P), 0, 0, 0, 62, 0, 1, ilog2(Mg)))) return st;
+        if ((st = a2a_())) return st;                   // (6) transpose P-major -> M-major
+        for (RankBufs& rb : p->ranks)                   //     [src][k2_local][k1_local] -> y[k1 + M k2]
+            for (int src = 0; src < p->G; ++src)
+                CUDA_TRY(cudaMemcpy2DAsync(out[gidx(rb)] + src * Mg, (size_t)p->M * sizeof(C), (const C*)rb.Rcv + src * rows * Mg,
+                                           (size_t)Mg * sizeof(C), (size_t)Mg * sizeof(C), (size_t)rows, cudaMemcpyDeviceToDevice, s));
+        return FMMFFT_SUCCESS;
+    }
+
     fmmfft_status_t run_forward() {
         fmmfft_status_t st;
-        if (p->direct) return mfft();
+        if (p->direct) return p->G > 1 ? run_direct_dist() : mfft(in[0]);
 #define STEP(stage, call) if ((st = mark(stage))) return st; if ((st = call)) return st;
         if ((st = mark(ST_COMM_S))) return st;
         if (p->G > 1) {                                 // S halo on the side stream (overlaps S2M)
@@ -1674,10 +1609,21 @@ fmmfft_status_t fmmfft_comm_destroy(void) {
 
 // FMMFFT_FLAG_DIRECT: the in-house Cooley-Tukey comparator — the same
 // four-step FFT kernels (k_fft_col + k_fft_rowt) on the whole length-N vector, no FMM.
+// FMMFFT_FLAG_DIRECT: the in-house Cooley-Tukey comparator — no FMM. G = 1: the
+// four-step FFT kernels (k_fft_col + k_fft_rowt) on the whole length-N vector. G > 1: the
+// distributed radix-P six-step FFT with its three all-to-alls, P = 2^ceil(log2 N / 2)
+// clamped to the column pass's range, the same exchange schedule (NCCL or virtual ranks).
 static fmmfft_status_t plan_direct(fmmfft_plan_t* plan, long long N, int G, fmmfft_precision_t precision, unsigned flags) {
     if (!pow2(N)) return fail(FMMFFT_INVALID_VALUE, "N must be a power of two");
-    if (G != 1) return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_DIRECT: single GPU only (G = 1)");
-    if (flags & (FMMFFT_FLAG_VIRTUAL | FMMFFT_FLAG_PROFILE)) return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_DIRECT: no virtual / profile");
+    if (!(G == 1 || G == 2 || G == 4 || G == 8)) return fail(FMMFFT_INVALID_VALUE, "G must be 1, 2, 4 or 8");
+    if (flags & FMMFFT_FLAG_PROFILE) return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_DIRECT: no profile");
+    const bool virt = (flags & FMMFFT_FLAG_VIRTUAL) != 0, vnccl = (flags & FMMFFT_FLAG_VIRTUAL_NCCL) != 0;
+    if (G == 1 && (virt || vnccl)) return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_DIRECT: virtual ranks need G > 1");
+    if (vnccl && !virt) return fail(FMMFFT_INVALID_VALUE, "FMMFFT_FLAG_VIRTUAL_NCCL needs FMMFFT_FLAG_VIRTUAL");
+    if ((G > 1 && !virt) || vnccl) {
+        if (!g_comm.comm) return fail(FMMFFT_NOT_INITIALIZED, "G > 1 needs fmmfft_comm_init");
+        if (g_comm.size != (vnccl ? 1 : G)) return fail(FMMFFT_INVALID_VALUE, "communicator size %d", g_comm.size);
+    }
     int dev = 0;
     CUDA_TRY(cudaGetDevice(&dev));
     cudaDeviceProp prop;
@@ -1685,19 +1631,51 @@ static fmmfft_status_t plan_direct(fmmfft_plan_t* plan, long long N, int G, fmmf
     if (prop.major != 10 || prop.minor != 0) return fail(FMMFFT_UNSUPPORTED, "sm_100a only");
     fmmfft_status_t st = precision == FMMFFT_C64 ? init_kernel_attrs<float>() : init_kernel_attrs<double>();
     if (st) return st;
+    const int lN = ilog2(N), lPmax = precision == FMMFFT_C64 ? 11 : 10;
+    const int lP = G == 1 ? 0 : std::max(5, std::min(lPmax, (lN + 1) / 2));
+    if (G > 1 && (lN - lP < 8 || (1LL << (lN - lP)) % G || (1LL << lP) % G || (N >> lP) / G < 16))
+        return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_DIRECT: N = 2^%d too small for G = %d", lN, G);
+    if (N / G > (1LL << 30)) return fail(FMMFFT_UNSUPPORTED, "N/G > 2^30 per rank not supported");
     fmmfft_plan_s* p = new fmmfft_plan_s;
-    p->N = N; p->M = N; p->Mg = N; p->P = 1; p->G = 1; p->prec = precision; p->flags = flags; p->device = dev;
-    p->direct = true;
+    p->N = N; p->P = 1 << lP; p->M = N >> lP; p->G = G; p->Mg = p->M / G; p->prec = precision; p->flags = flags;
+    p->device = dev; p->virt = virt; p->direct = true;
     p->inverse = (flags & FMMFFT_FLAG_INVERSE) != 0;
     p->esz = precision == FMMFFT_C64 ? 8 : 16;
     p->rsz = p->esz / 2;
-    choose_fourstep(p, ilog2(N), precision == FMMFFT_C64 ? 11 : 10);
-    if (!p->fs_lr) { delete p; return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_DIRECT: need 2^10 <= N <= 2^%d", precision == FMMFFT_C64 ? 33 : 30); }
+    if ((G > 1 && !virt) || vnccl) {
+        p->comm = g_comm.comm;
+        p->comm_rank = g_comm.rank;
+        p->vnccl = vnccl;
+        ++g_comm_plans;
+    }
+    if (G == 1) {
+        choose_fourstep(p, lN, lPmax);
+        if (!p->fs_lr) { destroy_plan(p); return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_DIRECT: need 2^10 <= N <= 2^%d", precision == FMMFFT_C64 ? 33 : 30); }
+    } else {
+        plan_mfft(p);
+        if (p->row_fft1) {                               // k_fft_row's twiddles w_M^u, u < M/16
+            std::vector<double> tw(2 * (p->M / 16));
+            for (long long u = 0; u < p->M / 16; ++u) {
+                tw[2 * u] = std::cos(2 * M_PI * (double)u / (double)p->M);
+                tw[2 * u + 1] = -std::sin(2 * M_PI * (double)u / (double)p->M);
+            }
+            st = precision == FMMFFT_C64 ? upload<float>(p, &p->twM, tw) : upload<double>(p, &p->twM, tw);
+        }
+    }
     const char* g_env = getenv("FMMFFT_NO_GRAPH");
     p->use_graph = !(g_env && g_env[0] == '1');
-    p->ranks.resize(1);
-    st = dalloc(p, &p->ranks[0].tmp, (size_t)N * p->esz);
-    if (!st && p->inverse) st = dalloc(p, &p->ranks[0].cin, (size_t)N * p->esz);
+    const int nr = virt ? G : 1;
+    const size_t nl = (size_t)(N / G) * p->esz;
+    p->ranks.resize(nr);
+    for (int g = 0; g < nr && !st; ++g) {
+        RankBufs& rb = p->ranks[g];
+        rb.g = virt ? g : p->comm_rank;
+        st = dalloc(p, &rb.tmp, nl);
+        if (!st && p->inverse) st = dalloc(p, &rb.cin, nl);
+        if (!st && G > 1) st = dalloc(p, &rb.W, nl);
+        if (!st && G > 1) st = dalloc(p, &rb.Rcv, nl);
+        if (!st && G > 1) st = dalloc(p, &rb.Tn, nl);
+    }
     if (!st) {
         cudaError_t e = cudaStreamCreateWithFlags(&p->cap_stream, cudaStreamNonBlocking);
         if (e != cudaSuccess) st = fail(FMMFFT_CUDA_ERROR, "stream setup: %s", cudaGetErrorString(e));
@@ -1773,17 +1751,11 @@ static fmmfft_status_t plan_complex(fmmfft_plan_t* plan, long long N, int P, int
         cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
         const size_t scratch = (((size_t)3 * Q) << (L > 0 ? L - 1 : 0)) * p->esz + (size_t)2 * Q * Q * p->rsz;
         p->tree_p = (G == 1) && ((long long)Q << L) <= 8LL * threads && tree_p_smem(p, threads) + scratch <= (size_t)optin;
-        if (const char* e = getenv("FMMFFT_TREE")) {
-            p->tree_p = p->tree_p && (e[0] == 'p' || e[0] == 'f' || e[0] == 'c');
-            p->tree_phased = e[0] == 'p';
-        }
-        // complex64, Q = 8 / 16: split each FMM's tree over a cluster of CL CTAs (k_tree_pc)
-        if (p->tree_p && !p->tree_phased && precision == FMMFFT_C64 && (Q == 16 || Q == 8)) {
-            int cl = 2;
-            if (const char* e = getenv("FMMFFT_TREE_CL")) cl = atoi(e);
-            if (const char* e = getenv("FMMFFT_TREE")) if (e[0] == 'f') cl = 1;
-            if ((cl == 2 || cl == 4) && (1 << B) >= cl && tree_pc_smem(p, cl) <= (size_t)optin) p->tree_cl = cl;
-        }
+        // FMMFFT_TREE=w: the per-level (wide-tree) kernels even where the fused far field fits
+        if (const char* e = getenv("FMMFFT_TREE")) p->tree_p = p->tree_p && e[0] != 'w';
+        // complex64, Q = 8 / 16: each FMM's tree on a cluster of 2 CTAs (k_tree_pc); else one CTA
+        // per FMM (k_tree_p)
+        if (p->tree_p && precision == FMMFFT_C64 && (Q == 16 || Q == 8) && tree_pc_smem(p, 2) <= (size_t)optin) p->tree_cl = 2;
     }
     // tensor-core S2T (k_s2t_tc, 3xTF32 on tcgen05) for complex64 with M_L = 64 and whole 128-box
     // tiles per rank; FMMFFT_S2T=simt selects the FFMA2 kernel (k_near_up) instead
@@ -1792,43 +1764,9 @@ static fmmfft_status_t plan_complex(fmmfft_plan_t* plan, long long N, int P, int
     // the cluster far field gathers M^L and scatters L^L one FMM (one p) at a time: keep both
     // p-major so those are contiguous runs (debug plans keep [b][q][p] for the stage buffers)
     p->pmaj = p->tree_p && p->tree_cl > 1 && L > B && !(flags & FMMFFT_FLAG_DEBUG);
-    if (const char* e = getenv("FMMFFT_PMAJ")) p->pmaj = p->pmaj && e[0] != '0';
-    if (const char* e = getenv("FMMFFT_DOWN")) p->lvl_off = e[0] == 't';
-    if (const char* e = getenv("FMMFFT_PP")) p->pp_old = e[0] == 't';
-    if (const char* e = getenv("FMMFFT_S2T_TPC")) p->s2t_tpc = std::max(0, atoi(e));
-    if (const char* e = getenv("FMMFFT_S2M_NBX")) p->s2m_nbx = atoi(e) == 1 ? 1 : 2;
-    if (const char* e = getenv("FMMFFT_S2M_PC")) { const int v = atoi(e); if (v == 8 || v == 16 || (v == 32 && precision == FMMFFT_C64)) p->s2m_pc = v; }
-    if (const char* e = getenv("FMMFFT_PP_MS")) { const int v = atoi(e); if (v >= 8 && v <= M_L && pow2(v)) p->pp_ms = v; }
     const char* g_env = getenv("FMMFFT_NO_GRAPH");
     p->use_graph = !(g_env && g_env[0] == '1');
-    plan_radices(p);
-    {
-        const int lM = ilog2(p->M);
-        const char* e = getenv("FMMFFT_ROWFFT");
-        p->row_fft1 = lM >= 8 && lM <= (precision == FMMFFT_C64 ? 14 : 13) && !(e && e[0] == '0');
-        // cluster rows (k_fft_rowc, FMMFFT_ROWFFT_CL=2|4): each row split over CL CTAs
-        const int kmax = precision == FMMFFT_C64 ? 13 : 12;
-        const long long rows = P / G;
-        int cl = 0;                      // measured slower than k_fft_row on cfg2 (opt-in)
-        (void)rows;
-        if (const char* c = getenv("FMMFFT_ROWFFT_CL")) cl = atoi(c);
-        if (cl == 4 && lM - 2 < 8) cl = 2;
-        if ((cl == 2 || cl == 4) && lM - ilog2(cl) >= 8 && lM - ilog2(cl) <= kmax && !(e && e[0] == '0')) p->row_cl = cl;
-    }
-    {   // rows longer than one CTA's shared memory: the four-step passes (FMMFFT_MFFT=pass keeps k_fft_pass)
-        const int lM = ilog2(p->M);
-        int mx = 10;                     // 11-bit passes (1 CTA per SM) measured slower than 3 passes of <= 10 bits
-        if (const char* nw = getenv("FMMFFT_FS_NARROW")) p->fs_narrow = nw[0] == '1';
-        if (p->fs_narrow) mx = precision == FMMFFT_C64 ? 11 : 10;
-        if (const char* b = getenv("FMMFFT_FS_MAXBITS")) mx = std::max(6, std::min(mx, atoi(b)));
-        const char* e = getenv("FMMFFT_MFFT");
-        const bool want = !(e && e[0] == 'p') && !(getenv("FMMFFT_ROWFFT") && getenv("FMMFFT_ROWFFT")[0] == '0');
-        // FMMFFT_MFFT=fs forces it; by default also rows of >= 2^13 points when there are fewer rows
-        // than SMs (k_fft_row would run one CTA per row on part of the GPU)
-        const bool few_rows = P / G < 148 && lM >= 13 && !getenv("FMMFFT_ROWFFT_CL") && !(e && e[0] == 'r');
-        if (want && ((e && e[0] == 'f' && lM >= 10) || few_rows)) { p->row_fft1 = false; p->row_cl = 0; }
-        if (want && !p->row_fft1 && !p->row_cl) choose_fourstep(p, lM, mx);
-    }
+    plan_mfft(p);
     st = precision == FMMFFT_C64 ? build_tables<float>(p) : build_tables<double>(p);
     if (!st) {
         const int nr = virt ? G : 1;
@@ -1994,8 +1932,8 @@ fmmfft_status_t fmmfft_get_info(fmmfft_plan_t p, fmmfft_info_t* info) {
     info->L = p->L; info->precision = p->prec; info->M = p->M; info->level_gather = p->lg;
     info->n_stages = ST_COUNT + 1; info->workspace_bytes = p->ws_bytes; info->kernels_per_execute = p->kernels;
     info->variant = (p->tree_p ? FMMFFT_VARIANT_TREE_FUSED : 0u) | (p->s2t_tc ? FMMFFT_VARIANT_S2T_TC : 0u) |
-                    ((p->row_fft1 || p->row_cl) ? FMMFFT_VARIANT_ROW_FFT1 : 0u) | (p->fs_lr ? FMMFFT_VARIANT_FOURSTEP : 0u) |
-                    (p->row_cl ? FMMFFT_VARIANT_ROW_CL : 0u) | (!p->tree_p && !p->lvl_off ? FMMFFT_VARIANT_DOWN_LVL : 0u) |
+                    (p->row_fft1 ? FMMFFT_VARIANT_ROW_FFT1 : 0u) | (p->fs_lr ? FMMFFT_VARIANT_FOURSTEP : 0u) |
+                    (!p->tree_p && !p->direct ? FMMFFT_VARIANT_DOWN_LVL : 0u) |
                     (p->pmaj ? FMMFFT_VARIANT_PMAJ : 0u);
     return FMMFFT_SUCCESS;
 }

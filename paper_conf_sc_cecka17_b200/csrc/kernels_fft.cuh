@@ -445,123 +445,13 @@ k_fft_row(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, const C2<R>* __
     static_assert(L0 + 12 >= LLEN, "k_fft_row: LLEN <= L0 + 12");
 }
 
-// ---------------------------------------------------------------------------------------------
-// k_fft_rowc: the M-point FFT of one row (§3 step 4) on a cluster of CL CTAs, M = CL K.
-// Four-step split m = m1 + CL m2, k = k2 + K k1 (m1, k1 < CL; m2, k2 < K):
-//     X[k2 + K k1] = sum_{m1} w_CL^{m1 k1} w_M^{m1 k2} [ sum_{m2} x[m1 + CL m2] w_K^{m2 k2} ].
-// CTA r: (1) loads the contiguous block x[r K, (r+1) K) (coalesced, through the all-to-all receive
-// layout like k_fft_pass); (2) gathers its decimated sequence x[r + CL m2] from the cluster's
-// blocks through distributed shared memory and runs the K-point Stockham FFT in shared memory
-// (radix R0 then radix 16, as k_fft_row; twiddles w_K^u = w_M^{CL u} from the same table),
-// multiplying the last stage's natural-order output by w_M^{r k2}; (3) takes k2 in
-// [r K/CL, (r+1) K/CL), reads the CL partial spectra of those k2 through DSMEM and finishes
-// with a radix-CL DFT, storing CL contiguous runs of the output row.
-// ---------------------------------------------------------------------------------------------
+// radix-E DFT in registers, E in {2, 4, 8, 16}
 template <int E, typename C> __device__ __forceinline__ void dft_small(C* v) {
     if constexpr (E == 2) dft2(v);
     else if constexpr (E == 4) dft4(v);
     else if constexpr (E == 8) dft8(v);
     else dft16(v);
 }
-
-template <typename R, int LK, int CL>
-__global__ void __cluster_dims__(CL, 1, 1) __launch_bounds__(1 << (LK - 4))
-k_fft_rowc(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, const C2<R>* __restrict__ twM,
-           int in_row, int lblk, int blk_stride) {
-    namespace cg = cooperative_groups;
-    using C = C2<R>;
-    constexpr int K = 1 << LK, NT = K >> 4;
-    constexpr int LCL = CL == 2 ? 1 : (CL == 4 ? 2 : 3);
-    constexpr int LM = LK + LCL, M = 1 << LM;
-    constexpr int L0 = (LK & 3) ? (LK & 3) : 4, R0 = 1 << L0, NB0 = 16 / R0;
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    C* x = reinterpret_cast<C*>(smem_raw);                        // [row_pad(K)]
-    C* tw = x + row_pad(K);                                       // [M/16]  w_M^u
-    C* twc = tw + M / 16;                                         // [16 CL] w_{16 CL}^e
-    cg::cluster_group cluster = cg::this_cluster();
-    const int r = (int)cluster.block_rank();
-    const int tid = threadIdx.x;
-    const size_t row = blockIdx.x / CL;
-    for (int u = tid; u < M / 16; u += NT) cp_async_elem(tw + u, twM + u);
-    for (int e = tid; e < 16 * CL; e += NT) twc[e] = twiddle<R>(e, 16 * CL);
-    cp_async_commit();
-    pdl_wait();
-    // (1) contiguous block r of the row
-    {
-        const C* xin = in + row * (size_t)in_row;
-        const int bmask = (1 << lblk) - 1;
-        C v[16];
-#pragma unroll
-        for (int u = 0; u < 16; ++u) {
-            const int m = r * K + tid + u * NT;
-            v[u] = ldg_c(xin + (size_t)(m >> lblk) * blk_stride + (m & bmask));
-        }
-#pragma unroll
-        for (int u = 0; u < 16; ++u) x[row_pad(tid + u * NT)] = v[u];
-    }
-    cp_async_wait_all();
-    cluster.sync();
-    // (2) stage 0 of the K-point FFT on the decimated sequence y[m2] = x[r + CL m2] (DSMEM gather)
-    C v[16];
-#pragma unroll
-    for (int b = 0; b < NB0; ++b) {
-        const int j = tid + b * NT;
-#pragma unroll
-        for (int t = 0; t < R0; ++t) {
-            const int g = r + CL * (j + t * (K / R0));
-            v[b * R0 + t] = *cluster.map_shared_rank(x + row_pad(g & (K - 1)), g >> LK);
-        }
-    }
-#pragma unroll
-    for (int b = 0; b < NB0; ++b) dft_small<R0>(v + b * R0);
-    cluster.sync();                                              // every gather done: x is free
-#pragma unroll
-    for (int b = 0; b < NB0; ++b) {
-        const int j = tid + b * NT;
-#pragma unroll
-        for (int t = 0; t < R0; ++t) x[row_pad(j * R0 + t)] = v[b * R0 + t];
-    }
-    __syncthreads();
-    // radix-16 stages; the last one (Ns = K/16) gives Z[k2], k2 = j + t K/16, natural order
-    auto stage = [&](auto lnsc) {
-        constexpr int LNS = decltype(lnsc)::value, NS = 1 << LNS;
-        const int j = tid, k = j & (NS - 1);
-#pragma unroll
-        for (int t = 0; t < 16; ++t) v[t] = x[row_pad(j + t * NT)];
-        twiddle_powers<16>(v, tw[(k << (LK - 4 - LNS)) * CL]);  // w_K^u = w_M^{CL u}
-        dft16(v);
-        __syncthreads();
-        if constexpr (LNS + 4 < LK) {
-#pragma unroll
-            for (int t = 0; t < 16; ++t) x[row_pad(((j - k) << 4) + k + t * NS)] = v[t];
-        } else {                                                  // Z'[k2] = Z[k2] w_M^{r k2}
-            const C wj = tw[r * j];                               // w_M^{r j}, r j < M/16
-#pragma unroll
-            for (int t = 0; t < 16; ++t)                          // w_M^{r t K/16} = w_{16 CL}^{r t}
-                x[row_pad(j + t * NT)] = cmul(v[t], t ? cmul(wj, twc[(r * t) & (16 * CL - 1)]) : wj);
-        }
-        __syncthreads();
-    };
-    if constexpr (L0 < LK) stage(std::integral_constant<int, L0>{});
-    if constexpr (L0 + 4 < LK) stage(std::integral_constant<int, L0 + 4>{});
-    if constexpr (L0 + 8 < LK) stage(std::integral_constant<int, L0 + 8>{});
-    static_assert(L0 + 12 >= LK, "k_fft_rowc: LK <= L0 + 12");
-    cluster.sync();                                              // every partial spectrum written
-    // (3) k2 in [r K/CL, (r+1) K/CL): radix-CL DFT across the cluster's spectra
-    C* y = out + (row << LM);
-#pragma unroll
-    for (int u = 0; u < 16 / CL; ++u) {
-        const int k2 = r * (K / CL) + tid + u * NT;
-        C w[CL];
-#pragma unroll
-        for (int m1 = 0; m1 < CL; ++m1) w[m1] = *cluster.map_shared_rank(x + row_pad(k2), m1);
-        dft_small<CL>(w);
-#pragma unroll
-        for (int k1 = 0; k1 < CL; ++k1) y[k2 + K * k1] = w[k1];
-    }
-    cluster.sync();                                              // remote reads done before exit
-}
-
 
 // ---------------------------------------------------------------------------------------------
 // Large M (rows that do not fit one CTA's shared memory): the M-point FFT (§3 step 4) as a
@@ -713,6 +603,56 @@ k_fft_rowt(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, long long M, i
     for (int t = 0; t < 16; ++t) y[(long long)(j + t * NT) << lrpr] = v[t];
 }
 
+
+// ---------------------------------------------------------------------------------------------
+// The distributed radix-P Cooley-Tukey FFT (the six steps of P:283-310; the
+// comparator that isolates the transposes the FMM-FFT saves): F_N = Pi_{M,P} (I_M x F_P) Pi_{P,M}
+// T_{P,M} (I_P x F_M) Pi_{M,P}, N = M P, x block-distributed in natural order (rank g holds
+// x[p + P m] for m in its block of M/G and every p).
+//
+// k_transpose_rc: step 1's local half, out[c][r] = in[r][c] for a rows x cols matrix (rank g's
+// [m_local][p] block -> [p][m_local], so the all-to-all chunk of rank r is the contiguous rows
+// p in r's block). 32 x 32 tiles through padded shared memory, coalesced both ways.
+// ---------------------------------------------------------------------------------------------
+template <typename R>
+__global__ void __launch_bounds__(256)
+k_transpose_rc(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, long long rows, long long cols) {
+    pdl_trigger();
+    __shared__ C2<R> t[32][33];
+    const long long r0 = (long long)blockIdx.y * 32, c0 = (long long)blockIdx.x * 32;
+    pdl_wait();
+    for (int k = threadIdx.y; k < 32; k += 8) {
+        const long long r = r0 + k, c = c0 + threadIdx.x;
+        if (r < rows && c < cols) t[k][threadIdx.x] = in[r * cols + c];
+    }
+    __syncthreads();
+    for (int k = threadIdx.y; k < 32; k += 8) {
+        const long long c = c0 + k, r = r0 + threadIdx.x;
+        if (r < rows && c < cols) out[c * rows + r] = t[threadIdx.x][k];
+    }
+}
+
+// ---------------------------------------------------------------------------------------------
+// k_twiddle_chunk: steps 3 + 4's local half. Rank g holds X[p_local][k1] (rows p = g P/G +
+// p_local, the M-point FFTs of step 2); multiplies by the twiddle T = w_N^{p k1} and writes the
+// all-to-all send layout [r][p_local][k1_local] (k1 = r M/G + k1_local). The angle is reduced
+// exactly in integers and evaluated in float64.
+// ---------------------------------------------------------------------------------------------
+template <typename R>
+__global__ void __launch_bounds__(256)
+k_twiddle_chunk(const C2<R>* __restrict__ X, C2<R>* __restrict__ W, long long M, int lMg, int lrows, long long p0, long long N) {
+    pdl_trigger();
+    pdl_wait();
+    const long long total = M << lrows, Mg = 1LL << lMg;
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    for (long long o = (long long)blockIdx.x * blockDim.x + threadIdx.x; o < total; o += stride) {
+        const long long kl = o & (Mg - 1), pl = (o >> lMg) & ((1LL << lrows) - 1), r = o >> (lMg + lrows);
+        const long long k1 = r * Mg + kl;
+        const C2<R> v = X[pl * M + k1];
+        const double2 w = twiddle_d(((p0 + pl) * k1) & (N - 1), N);
+        W[o] = C2<R>{(R)(w.x * (double)v.x - w.y * (double)v.y), (R)(w.x * (double)v.y + w.y * (double)v.x)};
+    }
+}
 
 // ---------------------------------------------------------------------------------------------
 // Inverse transform (§8(f) NEXT-1): F_N^{-1} x = conj(F_N conj(x)) / N (F_N^{-1} = F_N^H / N),

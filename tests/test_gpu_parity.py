@@ -307,14 +307,10 @@ def test_real_full_size_sampled(F):
 # ------------------------------------------------------------------ alternative kernel paths
 @pytest.mark.parametrize("env", [
     {"FMMFFT_S2T": "simt"},      # S2T on the FFMA2 SIMT kernel (k_near_up) instead of tcgen05
-    {"FMMFFT_TREE": "f"},        # far field fused in one per-FMM kernel (k_tree_pq)
-    {"FMMFFT_TREE_CL": "4"},     # far field on a cluster of 4 CTAs per FMM (k_tree_pc)
     {"FMMFFT_TREE": "w"},        # far field as wide per-level kernels (k_up, k_base, k_tree_down + k_m2l_lvl)
-    {"FMMFFT_TREE": "w", "FMMFFT_DOWN": "tree"},   # ... with every down level in k_tree_down
     {"FMMFFT_NO_GRAPH": "1"},    # eager launches instead of a CUDA graph
-    {"FMMFFT_ROWFFT": "0"},      # multi-pass M-point FFT (k_fft_pass) instead of k_fft_row(c)
-    {"FMMFFT_ROWFFT_CL": "0"},   # one CTA per M-point row (k_fft_row)
-    {"FMMFFT_ROWFFT_CL": "2"},   # a cluster of 2 CTAs per row (k_fft_rowc)
+    {"FMMFFT_MFFT": "pass"},     # multi-pass M-point FFT (k_fft_pass) instead of k_fft_row
+    {"FMMFFT_MFFT": "fs"},       # four-step M-point FFT (k_fft_col + k_fft_rowt) instead of k_fft_row
 ])
 @pytest.mark.parametrize("N,P,B,Q,G", [(1 << 20, 64, 2, 16, 1), (1 << 20, 64, 3, 16, 4)])
 def test_alternative_paths(F, monkeypatch, env, N, P, B, Q, G):
@@ -385,10 +381,30 @@ def test_direct_fft(F, N, prec, inverse):
     assert rel(y, ref) < (1e-6 if prec == "c64" else 1e-13)
 
 
-def test_direct_rejects_multi_gpu(F):
-    from paper_conf_sc_cecka17_b200._lib import FmmfftError
-    with pytest.raises(FmmfftError):
-        F(N=1 << 20, P=2, G=2, virtual=True, direct=True)
+@pytest.mark.parametrize("N,G,prec,inverse", [
+    (1 << 20, 2, "c64", False), (1 << 22, 4, "c64", False), (1 << 24, 8, "c64", False),
+    (1 << 18, 8, "c128", False), (1 << 21, 4, "c128", True), (1 << 16, 2, "c64", True),
+])
+def test_direct_distributed(F, N, G, prec, inverse):
+    """The distributed radix-P Cooley-Tukey FFT with three all-to-alls (NEXT-3) through
+    virtual ranks: every element against the float64 DFT."""
+    x = SI.complex_uniform(0, N, dtype=NPDT[prec])
+    plan = F(N=N, P=1, G=G, precision=prec, direct=True, virtual=True, inverse=inverse)
+    y = plan(torch.from_numpy(x).cuda()).cpu().numpy()
+    ref = O.fft_radix2(x, inverse=inverse)
+    assert rel(y, ref) < (1e-6 if prec == "c64" else 1e-13)
+
+
+def test_direct_distributed_nccl_transport(F, nccl_local):
+    N, G = 1 << 20, 4
+    x = torch.from_numpy(SI.complex_uniform(0, N, dtype=np.complex64)).cuda()
+    a = F(N=N, P=1, G=G, precision="c64", direct=True, virtual=True, transport="nccl")
+    b = F(N=N, P=1, G=G, precision="c64", direct=True, virtual=True)
+    ya, yb = a(x), b(x)
+    torch.cuda.synchronize()
+    assert torch.equal(ya, yb)
+    a.close()
+    b.close()
 
 
 # ------------------------------------------------------------------ autotuner, measured (§8(f) NEXT-2)
@@ -411,12 +427,10 @@ def test_autotune_c128_meets_tol(F, N):
     assert rel(y, O.fft_radix2(x)) < 1e-11
 
 
-@pytest.mark.parametrize("env", [None, {"FMMFFT_PP": "tile"}])
-@pytest.mark.parametrize("P,Q,prec", [(16, 16, "c64"), (32, 8, "c64"), (8, 24, "c128"), (2, 16, "c64"), (64, 16, "c64"), (64, 24, "c128")])
-def test_post_pfft_variants(F, monkeypatch, env, P, Q, prec):
-    """k_post_pfft_r (P <= 32, registers) and the shared-memory-tile k_post_pfft agree with the oracle."""
-    for k, v in (env or {}).items():
-        monkeypatch.setenv(k, v)
+@pytest.mark.parametrize("P,Q,prec", [(16, 16, "c64"), (32, 8, "c64"), (8, 24, "c128"), (2, 16, "c64"), (64, 16, "c64"),
+                                       (64, 24, "c128"), (128, 16, "c64")])
+def test_post_pfft_variants(F, P, Q, prec):
+    """k_post_pfft_r (P <= 32, registers) and the shared-memory-tile k_post_pfft (P > 32) agree with the oracle."""
     N = 1 << 18
     plan, x, y = run(F, N, P, 2, Q, prec, 64)
     assert rel(y, O.fft_radix2(x)) < (1e-5 if prec == "c64" else 1e-11)
