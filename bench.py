@@ -494,6 +494,29 @@ print(json.dumps({"rc": rc, "err": err.value.decode(), "ms": [ms[0], ms[1]]}))
     return out
 
 
+def inhouse_3transpose(N, prec, world, x, flush, steps, stream, barrier):
+    """The library's own distributed radix-P Cooley-Tukey FFT with THREE all-to-alls
+    (FMMFFT_FLAG_DIRECT at G > 1): same N, same shards, same
+    exchange code and M-FFT kernels as the FMM-FFT, so the ratio isolates the transposes saved."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_cecka17_b200 import FmmFFT
+    d = FmmFFT(N=N, P=1, G=world, precision=prec, direct=True)
+    y = torch.empty_like(x)
+    for _ in range(3):
+        d(x, y, stream)
+    torch.cuda.synchronize()
+    barrier()
+    ms = statistics.median(timed_steps(lambda: d(x, y, stream), flush, steps, stream))
+    barrier()
+    t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    d.close()
+    return {"value": flops_fft(N) / (float(t) * 1e-3) / 1e9, "unit": "GFLOP/s", "ms_per_step": float(t),
+            "kernels": "k_transpose_rc, k_fft_col + k_fft_rowt, k_twiddle_chunk, k_fft_col + 3 NCCL all-to-alls"}
+
+
 def autotuned_pick(N, prec, flush, steps, x, stream):
     import torch
     from paper_conf_sc_cecka17_b200 import FmmFFT, autotune
@@ -585,6 +608,10 @@ def run_fmmfft(args, rank, world, local_rank):
                 "parseval_rel_dev": c2["parseval_rel_dev"], "kernels_per_execute": c2["info"]["kernels_per_execute"]}}
             c2["plan"].close()
     if world > 1 and not args.no_extras:
+        try:
+            extras["inhouse_3transpose"] = inhouse_3transpose(N, prec, world, res["x"], flush, comp_steps, stream, barrier)
+        except Exception as e:  # context only
+            extras["inhouse_3transpose"] = {"error": str(e)[:200]}
         yb = res["y"].cpu().numpy() if rank == 0 else None
         if rank == 0:
             extras["comparator"] = cufftxt_comparator(N, prec, world, comp_steps, yb)
