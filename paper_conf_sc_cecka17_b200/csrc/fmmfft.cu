@@ -348,7 +348,7 @@ static fmmfft_status_t build_tables(fmmfft_plan_s* p) {
                             cotpi((z[j] / 2 - z[i] / 2 + s) / (double)(1LL << lev) + (double)pp / (double)N);
         }
         if ((st = upload<R>(p, base ? &p->m2lB : &p->m2l[lev], t))) return st;
-        if (p->tree_p) {                                   // [p][s][j][i] (i fastest) for k_tree_p
+        {                                                  // [p][s][j][i] (i fastest): k_tree_p*, k_down_narrow
             std::vector<double> tp((size_t)P * ns * Q * Q, 0.0);
             for (int pp = 0; pp < P; ++pp)
                 for (int si = 0; si < ns; ++si)
@@ -570,6 +570,12 @@ static fmmfft_status_t init_kernel_attrs() {
                 set((const void*)k_post_pfft_r<R, decltype(v)::value, 16>);
                 set((const void*)k_post_pfft_r<R, decltype(v)::value, 24>);
             });
+        set((const void*)k_up_narrow<R, 8>);
+        set((const void*)k_up_narrow<R, 16>);
+        set((const void*)k_up_narrow<R, 24>);
+        set((const void*)k_down_narrow<R, 8>);
+        set((const void*)k_down_narrow<R, 16>);
+        set((const void*)k_down_narrow<R, 24>);
         set((const void*)k_m2l_lvl<R, 8>);
         set((const void*)k_m2m_lvl<R, 8>);
         set((const void*)k_m2m_lvl<R, 16>);
@@ -914,6 +920,18 @@ struct Exec {
             nbc >>= 1;
             --cur;
         }
+        if (cur > to && narrow_ok() && narrow_up_fits(nbc)) {   // every remaining level in one launch
+            NarrowUp no{};
+            for (int l = to; l < cur; ++l) no.out[l] = outs(l);
+            const size_t smem = narrow_up_smem((int)nbc);
+            dispatch<8, 16, 24>(p->Q, [&](auto qv) {
+                constexpr int QV = decltype(qv)::value;
+                launch_pdl(k_up_narrow<R, QV>, (unsigned)p->P, 256, smem, s, src, no, cur - 1, to, (int)nbc,
+                           (const R*)p->m2m, p->P);
+            });
+            LAUNCH_CHECK();
+            return FMMFFT_SUCCESS;
+        }
         while (cur > to) {
             int h = std::min(4, cur - to);
             while ((1LL << h) > nbc) --h;
@@ -931,6 +949,19 @@ struct Exec {
             cur -= h;
         }
         return FMMFFT_SUCCESS;
+    }
+
+    // k_up_narrow / k_down_narrow keep a whole narrow subtree of one FMM on chip (<= 200 KB)
+    bool narrow_ok() const { return p->Q == 8 || p->Q == 16 || p->Q == 24; }
+    bool narrow_up_fits(long long nin) const { return nin <= 1024 && narrow_up_smem((int)nin) <= 200 * 1024; }
+    bool narrow_down_fits(long long nmax) const { return nmax <= 1024 && narrow_down_smem((int)nmax) <= 200 * 1024; }
+    size_t narrow_down_smem(int nmax) const {
+        const size_t bsc = (size_t)(2 * p->Q + 2) / 2;
+        return (size_t)10 * p->Q * p->Q * sizeof(R) + ((size_t)4 * (nmax / 2 + 2) + 2 * (size_t)nmax) * bsc * sizeof(C);
+    }
+    size_t narrow_up_smem(int nin) const {
+        const size_t bsc = (size_t)(2 * p->Q + 2) / 2;
+        return (size_t)2 * p->Q * p->Q * sizeof(R) + ((size_t)nin + nin / 2) * bsc * sizeof(C);
     }
 
     // ---- the whole far field per FMM p in one launch (G = 1): M2M, M2L-B, REDUCE, M2L + L2L
@@ -1089,9 +1120,53 @@ struct Exec {
 
     // ---- down: M2L + L2L for every level B+1 .. L: k_tree_down over the upper levels (one
     // launch, per leaf range), then one k_m2l_lvl launch per wide level
+    // targets of level lev on this rank: all 2^lev boxes (G = 1, or the replicated levels < l_g),
+    // else the rank's own boxes
+    std::pair<long long, int> narrow_targets(long long g, int lev) const {
+        if (p->G == 1 || lev < p->lg) return {0, 1 << lev};
+        return {g * nb_at(lev), nb_at(lev)};
+    }
+
     fmmfft_status_t down() {
         if (p->L == p->B || p->tree_p) return FMMFFT_SUCCESS;
-        const int lnew = lvl_first();
+        int lnew = lvl_first();
+        if (narrow_ok()) {                           // k_down_narrow up to the widest level that fits
+            int lnar = p->B, nmax = 0;
+            for (int lev = p->B + 1; lev < lnew; ++lev) {
+                const int n = narrow_targets(0, lev).second;
+                if (!narrow_down_fits(std::max(nmax, n))) break;
+                nmax = std::max(nmax, n);
+                lnar = lev;
+            }
+            constexpr int PCl = lvl_pc<R>();
+            const bool lvl_usable = p->PCd % PCl == 0 && p->P % PCl == 0;
+            if (lnar > p->B && lnar == lnew - 1 && (lnar == p->L || lvl_usable)) {   // every narrow level
+                for (RankBufs& rb : p->ranks) {
+                    const long long g = grank(rb);
+                    NarrowArgs na{};
+                    for (int lev = p->B + 1; lev <= lnar; ++lev) {
+                        const TreeLevel tl = level_io(rb, lev, g);
+                        NarrowLevel& nl = na.lev[lev];
+                        nl.src = tl.src; nl.src_base = tl.src_base; nl.src_mod = tl.src_mod;
+                        nl.tab = p->m2l_pmaj[lev]; nl.out = tl.out; nl.out_base = tl.out_base;
+                        const auto ft = narrow_targets(g, lev);
+                        nl.f = ft.first; nl.n = ft.second;
+                    }
+                    if (p->lg == p->B) { na.par0 = rb.Lloc[p->B]; na.par0_base = g * nb_at(p->B); }
+                    else { na.par0 = rb.Lfull[p->B]; na.par0_base = 0; }
+                    na.lstart = p->B + 1;
+                    na.Lv = lnar;
+                    na.nmax = nmax;
+                    dispatch<8, 16, 24>(p->Q, [&](auto qv) {
+                        constexpr int QV = decltype(qv)::value;
+                        launch_pdl(k_down_narrow<R, QV>, (unsigned)(p->P - 1), 256, narrow_down_smem(nmax), s, na,
+                                   (const R*)p->m2m, p->P);
+                    });
+                    LAUNCH_CHECK();
+                }
+                return down_levels(lnar + 1);
+            }
+        }
         const int Lv = lnew - 1;                     // k_tree_down's (virtual) leaf level
         const int PC_ = p->PCd;
         const int npc = p->P / PC_;
@@ -1129,7 +1204,17 @@ struct Exec {
                 });
                 LAUNCH_CHECK();
             }
-            for (int lev = lnew; lev <= p->L; ++lev) {
+        }
+        return down_levels(lnew);
+    }
+
+    // one k_m2l_lvl launch per level first..L (wide levels: M2L + L2L, register-blocked)
+    fmmfft_status_t down_levels(int first) {
+        int optin = 0;
+        CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, p->device));
+        for (RankBufs& rb : p->ranks) {
+            const long long g = grank(rb);
+            for (int lev = first; lev <= p->L; ++lev) {
                 const TreeLevel tl = level_io(rb, lev, g);
                 LvlArgs la{};
                 la.src = tl.src; la.src_base = tl.src_base; la.src_mod = tl.src_mod;
