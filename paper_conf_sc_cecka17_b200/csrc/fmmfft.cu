@@ -198,6 +198,7 @@ struct RankBufs {
     void* haloL = nullptr;   // S box -1  (G > 1)
     void* haloR = nullptr;   // S box nb  (G > 1)
     void* r = nullptr;       // [P] reductions
+    void* dc = nullptr;      // [P/G] the k1 = 0 outputs of this rank's M-FFT rows (k_dc_bins, R19)
     void* cin = nullptr;     // conj(in) (inverse plans)
     void* rz = nullptr;      // Z = F_{N/2} z (real-input plans, FMMFFT_FLAG_REAL)
     void* din = nullptr;     // execute_host staging
@@ -254,6 +255,7 @@ struct fmmfft_plan_s {
     cudaEvent_t fork2 = nullptr;     // S' ready (tensor-core S2T)
     cudaStream_t side = nullptr;     // S2T runs here, concurrently with the far field
     cudaEvent_t cs_done = nullptr;   // S halo exchange (side stream) complete: orders NCCL work
+    cudaEvent_t dc_fork = nullptr, dc_join = nullptr;   // k_dc_bins on the side stream (after top)
     ncclComm_t comm = nullptr;       // G > 1 (non-virtual): the communicator, bound at plan time;
                                      // virtual + FMMFFT_FLAG_VIRTUAL_NCCL: a 1-rank communicator
     int comm_rank = 0;
@@ -478,6 +480,7 @@ static fmmfft_status_t alloc_rank(fmmfft_plan_s* p, RankBufs& rb) {
         if ((st = dalloc(p, &rb.haloR, (size_t)p->M_L * p->P * e))) return st;
     }
     if ((st = dalloc(p, &rb.r, (size_t)p->P * e))) return st;
+    if ((st = dalloc(p, &rb.dc, (size_t)(p->P / p->G) * e))) return st;
     rb.Mpad.assign(p->L + 1, nullptr);
     rb.Lloc.assign(p->L + 1, nullptr);
     rb.Mfull.assign(p->L + 1, nullptr);
@@ -510,6 +513,8 @@ static void destroy_plan(fmmfft_plan_s* p) {
     if (p->join) cudaEventDestroy(p->join);
     if (p->fork2) cudaEventDestroy(p->fork2);
     if (p->cs_done) cudaEventDestroy(p->cs_done);
+    if (p->dc_fork) cudaEventDestroy(p->dc_fork);
+    if (p->dc_join) cudaEventDestroy(p->dc_join);
     if (p->comm) --g_comm_plans;
     if (p->side) cudaStreamDestroy(p->side);
     if (p->cap_stream) cudaStreamDestroy(p->cap_stream);
@@ -1328,6 +1333,7 @@ struct Exec {
         const int lM = ilog2(p->M);
         for (RankBufs& rb : p->ranks) {
             C* dst = to_tn ? (C*)rb.Tn : out[gidx(rb)];
+            const C* dcp = p->direct ? nullptr : (const C*)rb.dc;    // the rows' k = 0 outputs (R19)
             const C* src = src_override ? src_override : (const C*)(p->G > 1 ? rb.Rcv : rb.W);
             if (src_override == in[0] && p->virt) src = in[gidx(rb)];
             long long in_row = p->M, blk_stride = 0;
@@ -1350,7 +1356,7 @@ struct Exec {
                     constexpr int CR = fs_cols<R>(LL);
                     if constexpr (LL <= fs_max<R>())
                         launch_pdl(k_fft_rowt<R, LL, CR>, (unsigned)(trows / CR), CR << (LL - 4), fft_rowt_smem<R, LL, CR>(), s,
-                                   bsrc, dst, (long long)p->M, lrpr);
+                                   bsrc, dst, (long long)p->M, lrpr, dcp);
                 });
                 if (!ok) return fail(FMMFFT_UNSUPPORTED, "k_fft_rowt: 2^%d", p->fs_lr);
                 LAUNCH_CHECK();
@@ -1362,7 +1368,7 @@ struct Exec {
                     constexpr int LL = decltype(ll)::value;
                     if constexpr (LL <= kRowFftMax<R>)
                         launch_pdl(k_fft_row<R, LL>, (unsigned)rows, 1 << (LL - 4), smem, s, src, dst, (const C*)p->twM,
-                                   (int)in_row, lblk == 62 ? lM : lblk, (int)blk_stride);
+                                   (int)in_row, lblk == 62 ? lM : lblk, (int)blk_stride, dcp);
                 });
                 LAUNCH_CHECK();
                 continue;
@@ -1384,7 +1390,8 @@ struct Exec {
                 const dim3 grid((unsigned)(nj / c), (unsigned)rows);
                 dispatch<1, 2, 3, 4, 5, 6, 7, 8, 9, 10>(lR, [&](auto lr) {
                     constexpr int LR = decltype(lr)::value;
-                    launch_pdl(k_fft_pass<R, LR>, grid, threads, smem, s, src, o, lM, lNs, ilog2(c), ir, lb, bs);
+                    launch_pdl(k_fft_pass<R, LR>, grid, threads, smem, s, src, o, lM, lNs, ilog2(c), ir, lb, bs,
+                               i == n - 1 ? dcp : (const C*)nullptr);
                 });
                 LAUNCH_CHECK();
                 src = o;
@@ -1394,9 +1401,12 @@ struct Exec {
         return FMMFFT_SUCCESS;
     }
 
-    // the k1 = 0 bins of the local M-FFT rows from the reductions r_p (k_dc_bins, reading R19)
+    // the k1 = 0 bins of the local M-FFT rows from the reductions r_p (k_dc_bins, reading R19): on
+    // the side stream once r is known (after top), into rb.dc; the last M-FFT pass stores them
     fmmfft_status_t dc_bins() {
         const int rows = p->P / p->G;
+        CUDA_TRY(cudaEventRecord(p->dc_fork, s));
+        CUDA_TRY(cudaStreamWaitEvent(side(), p->dc_fork, 0));
         for (RankBufs& rb : p->ranks) {
             // r_0: reduced by the per-level kernels (k_base*), or here from M^L's slot 0 when the
             // fused per-FMM far field (p = 1..P-1 only) ran
@@ -1407,10 +1417,11 @@ struct Exec {
                 m0_n = (long long)p->nb * p->Q;
                 m0_stride = p->pmaj ? 1 : p->P;
             }
-            launch_pdl(k_dc_bins<R>, (unsigned)((rows + 7) / 8), 256, 0, s, out[gidx(rb)], (const C*)rb.r, m0, m0_n,
+            launch_pdl(k_dc_bins<R>, (unsigned)((rows + 7) / 8), 256, 0, side(), (C*)rb.dc, (const C*)rb.r, m0, m0_n,
                        m0_stride, p->P, rows, grank(rb) * rows, (long long)p->M);
             LAUNCH_CHECK();
         }
+        CUDA_TRY(cudaEventRecord(p->dc_join, side()));
         return FMMFFT_SUCCESS;
     }
 
@@ -1511,12 +1522,14 @@ struct Exec {
         STEP(ST_M2M, m2m_local())
         STEP(ST_COMM_M, comm_M())
         STEP(ST_TOP, top())
+        if ((st = dc_bins())) return st;
         STEP(ST_DOWN, down())
         if ((st = join_near())) return st;
         STEP(ST_PFFT, post_pfft())
         STEP(ST_A2A, a2a())
-        STEP(ST_MFFT, mfft())
-        if ((st = dc_bins())) return st;
+        if ((st = mark(ST_MFFT))) return st;
+        CUDA_TRY(cudaStreamWaitEvent(s, p->dc_join, 0));
+        if ((st = mfft())) return st;
 #undef STEP
         return mark(ST_COUNT);
     }
@@ -1878,6 +1891,8 @@ static fmmfft_status_t plan_complex(fmmfft_plan_t* plan, long long N, int P, int
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->join, cudaEventDisableTiming);
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->fork2, cudaEventDisableTiming);
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->cs_done, cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->dc_fork, cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->dc_join, cudaEventDisableTiming);
         if (e == cudaSuccess && (flags & FMMFFT_FLAG_PROFILE)) {
             e = cudaEventCreate(&p->ev_s2t[0]);
             if (e == cudaSuccess) e = cudaEventCreate(&p->ev_s2t[1]);

@@ -251,7 +251,7 @@ k_post_pfft(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2
 template <typename R, int LR>
 __global__ void __launch_bounds__(sizeof(R) == 4 ? 1024 : 512)
 k_fft_pass(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, int lM, int lNs, int lc,
-           int in_row, int lblk, int blk_stride) {
+           int in_row, int lblk, int blk_stride, const C2<R>* __restrict__ dc) {
     pdl_trigger();
     using C = C2<R>;
     constexpr int Rp = 1 << LR, LD = Rp + 1;
@@ -310,6 +310,10 @@ k_fft_pass(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, int lM, int lN
             const int t = rem >> lNs, k = rem & (Ns - 1);
             yout[(j0 << LR) + idx] = tile[((jb << lNs) + k) * LD + t];
         }
+    }
+    if (dc != nullptr && j0 == 0) {                              // the row's k = 0 output (R19)
+        __syncthreads();
+        if (tid == 0) yout[0] = dc[row];
     }
 }
 
@@ -385,7 +389,7 @@ __device__ __forceinline__ constexpr int row_pad(int a) { return a + (a >> 4); }
 template <typename R, int LLEN>
 __global__ void __launch_bounds__(1 << (LLEN - 4))
 k_fft_row(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, const C2<R>* __restrict__ twM,
-          int in_row, int lblk, int blk_stride) {
+          int in_row, int lblk, int blk_stride, const C2<R>* __restrict__ dc) {
     using C = C2<R>;
     constexpr int M = 1 << LLEN, NT = M >> 4;
     constexpr int L0 = (LLEN & 3) ? (LLEN & 3) : 4, R0 = 1 << L0, NB0 = 16 / R0;
@@ -443,6 +447,10 @@ k_fft_row(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, const C2<R>* __
     if constexpr (L0 + 4 < LLEN) stage(std::integral_constant<int, L0 + 4>{});
     if constexpr (L0 + 8 < LLEN) stage(std::integral_constant<int, L0 + 8>{});
     static_assert(L0 + 12 >= LLEN, "k_fft_row: LLEN <= L0 + 12");
+    if (dc != nullptr) {                                         // the row's k = 0 output (R19)
+        __syncthreads();
+        if (threadIdx.x == 0) out[(size_t)blockIdx.x << LLEN] = dc[blockIdx.x];
+    }
 }
 
 // radix-E DFT in registers, E in {2, 4, 8, 16}
@@ -553,7 +561,7 @@ template <typename R, int LL, int CR> __host__ __device__ constexpr size_t fft_r
 
 template <typename R, int LL, int CR>
 __global__ void __launch_bounds__(CR << (LL - 4))
-k_fft_rowt(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, long long M, int lrpr) {
+k_fft_rowt(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, long long M, int lrpr, const C2<R>* __restrict__ dc) {
     pdl_trigger();
     using C = C2<R>;
     constexpr int Mr = 1 << LL, NT = Mr >> 4, CS = col_stride<Mr, CR>();
@@ -601,6 +609,10 @@ k_fft_rowt(const C2<R>* __restrict__ in, C2<R>* __restrict__ out, long long M, i
     C* y = out + row * M + pre;
 #pragma unroll
     for (int t = 0; t < 16; ++t) y[(long long)(j + t * NT) << lrpr] = v[t];
+    if (dc != nullptr && (r0 & ((1LL << lrpr) - 1)) == 0) {     // this CTA holds the row's k = 0 output (R19)
+        __syncthreads();
+        if (tid == 0) out[(r0 >> lrpr) * M] = dc[r0 >> lrpr];
+    }
 }
 
 
@@ -686,7 +698,9 @@ k_conj_scale(const C2<R>* in, C2<R>* out, long long n, R scale) {   // in == out
 // error at M = 2^22 (growing like sqrt M) while every other bin is at ~1e-6; the reductions r_p of
 // Algorithm 1 line 11 hold the same quantities accurately. r_0 (p = 0 is no FMM) is
 // the sum of M^L's slot 0 (S2M columns sum to 1): read from r[0] when the level kernels reduced it,
-// else reduced here from M^L slot 0 (m0: m0_n values at stride m0_stride). Sums in float64.
+// else reduced here from M^L slot 0 (m0: m0_n values at stride m0_stride). Sums in float64. Writes
+// dc[row] for this rank's rows; the last M-FFT pass (k_fft_rowt / k_fft_row / k_fft_pass) stores
+// dc[row] as the row's k1 = 0 output, so this kernel runs off the critical path (side stream).
 // ---------------------------------------------------------------------------------------------
 template <typename R>
 __global__ void __launch_bounds__(256)
@@ -702,10 +716,15 @@ k_dc_bins(C2<R>* __restrict__ y, const C2<R>* __restrict__ r, const C2<R>* __res
     for (int j = tid; j < P; j += blockDim.x) rr[j] = make_double2((double)r[j].x, (double)r[j].y);
     if (m0 != nullptr) {                                          // r_0 = sum of M^L slot 0
         double2 a = make_double2(0.0, 0.0);
-        for (long long i = tid; i < m0_n; i += blockDim.x) {
-            const C2<R> v = m0[i * m0_stride];
-            a.x += (double)v.x;
-            a.y += (double)v.y;
+        for (long long i0 = tid; i0 < m0_n; i0 += 8LL * blockDim.x) {   // 8 independent loads in flight
+            C2<R> v[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+                const long long i = i0 + (long long)u * blockDim.x;
+                v[u] = i < m0_n ? m0[i * m0_stride] : C2<R>{R(0), R(0)};
+            }
+#pragma unroll
+            for (int u = 0; u < 8; ++u) { a.x += (double)v[u].x; a.y += (double)v[u].y; }
         }
         for (int o = 16; o > 0; o >>= 1) {                        // fixed-order reduction: deterministic
             a.x += __shfl_xor_sync(0xffffffffu, a.x, o);
@@ -734,7 +753,7 @@ k_dc_bins(C2<R>* __restrict__ y, const C2<R>* __restrict__ r, const C2<R>* __res
         acc.x += __shfl_xor_sync(0xffffffffu, acc.x, o);
         acc.y += __shfl_xor_sync(0xffffffffu, acc.y, o);
     }
-    if (lane == 0) y[(size_t)row * M] = C2<R>{(R)acc.x, (R)acc.y};
+    if (lane == 0) y[row] = C2<R>{(R)acc.x, (R)acc.y};
 }
 
 // ---------------------------------------------------------------------------------------------

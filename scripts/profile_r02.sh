@@ -21,7 +21,8 @@ PY
   per=$(( n / 15 ))  # --steps 2 --warmup 3: 5 executes each of the timed, profiled and e2e plans; capture the 3rd
   timeout 1200 ncu --set full --metrics $EXTRA --clock-control none --import-source on -k regex:"k_" --launch-skip $(( 2 * per )) -c $per \
       -o /tmp/full_$w python bench.py --workload $w --steps 1 --warmup 3 --no-cpu-baseline --no-extras > /dev/null 2>&1
-  python scripts/ncu_traffic.py /tmp/full_$w.ncu-rep ${w}_G1 gpurun_out/prof/${tag}_ncu_full_$w.txt > /dev/null
+  key=${w}_G1; [ "$w" = cfg3v8 ] && key=cfg3v8_G8
+  python scripts/ncu_traffic.py /tmp/full_$w.ncu-rep $key gpurun_out/prof/${tag}_ncu_full_$w.txt > /dev/null
   ncu -i /tmp/full_$w.ncu-rep --page details --csv 2>/dev/null | gzip > gpurun_out/prof/${tag}_details_$w.csv.gz
 done
 python scripts/sass_evidence.py paper_conf_sc_cecka17_b200/libfmmfft.so > gpurun_out/prof/${tag}_sass_tcgen05.txt
