@@ -7,7 +7,7 @@ import ctypes
 import os
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libfmmfft.so")
+LIB_PATH = os.environ.get("FMMFFT_LIB") or os.path.join(_PKG, "libfmmfft.so")   # FMMFFT_LIB: a tuning build
 
 SUCCESS, INVALID_VALUE, UNSUPPORTED, ALLOC_FAILED, CUDA_ERROR, NCCL_ERROR, NOT_INITIALIZED = range(7)
 STATUS_NAMES = ["SUCCESS", "INVALID_VALUE", "UNSUPPORTED", "ALLOC_FAILED", "CUDA_ERROR", "NCCL_ERROR",

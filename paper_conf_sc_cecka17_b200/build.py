@@ -64,6 +64,18 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB
 
 
+def build_variant(name: str, defines) -> str:
+    """A tuning build with extra -D macros: paper_conf_sc_cecka17_b200/libfmmfft_<name>.so (select it
+    with FMMFFT_LIB=<path>; the default library is unaffected)."""
+    out = os.path.join(PKG, f"libfmmfft_{name}.so")
+    cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
+           "-Xcompiler", "-fvisibility=hidden", "--expt-relaxed-constexpr", "--split-compile=8",
+           *[f"-D{d}" for d in defines], "-I", os.path.join(ROOT, "include"), "-I", _nccl_include(),
+           os.path.join(CSRC, "fmmfft.cu"), "-o", out, "-ldl"]
+    subprocess.run(cmd, check=True)
+    return out
+
+
 CMP_SRC = os.path.join(ROOT, "comparators", "cufftxt.cu")
 CMP_LIB = os.path.join(ROOT, "comparators", "libcufftxt_cmp.so")
 

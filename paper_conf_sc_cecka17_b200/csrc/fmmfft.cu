@@ -461,7 +461,10 @@ static void plan_mfft(fmmfft_plan_s* p) {
     const bool few_rows = p->P / p->G < 148 && lM >= 13;
     if ((fs && lM >= 10) || few_rows) p->row_fft1 = false;
     // 11-bit passes (1 CTA per SM) measured slower than 3 passes of <= 10 bits
-    if (!pass && !p->row_fft1) choose_fourstep(p, lM, 10);
+#ifndef FMMFFT_FS_MX
+#define FMMFFT_FS_MX 10
+#endif
+    if (!pass && !p->row_fft1) choose_fourstep(p, lM, FMMFFT_FS_MX);
 }
 
 static fmmfft_status_t alloc_rank(fmmfft_plan_s* p, RankBufs& rb) {
@@ -521,6 +524,10 @@ static void destroy_plan(fmmfft_plan_s* p) {
     delete p;
 }
 
+#ifndef FMMFFT_NEAR_IB_D
+#define FMMFFT_NEAR_IB_D 8           // complex128 k_near_up: outputs per thread (register block)
+#endif
+
 // Raise every kernel's dynamic shared memory cap once per device (function attributes are
 // per device; not legal during capture). Called with the plan's device current.
 template <typename R>
@@ -543,7 +550,7 @@ static fmmfft_status_t init_kernel_attrs() {
                 e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, optin - (int)fa.sharedSizeBytes);
             if (e != cudaSuccess && err == cudaSuccess) err = e;
         };
-        constexpr int IB = sizeof(R) == 4 ? 16 : 8;
+        constexpr int IB = sizeof(R) == 4 ? 16 : FMMFFT_NEAR_IB_D;
         auto per_pc = [&](auto pc) {
             constexpr int PCv = decltype(pc)::value;
             set((const void*)k_near_up<R, IB, PCv>);
@@ -646,7 +653,7 @@ struct Exec {
     std::vector<C*> out;
     int nlaunch = 0;             // kernels launched by this execute (all virtual ranks)
 
-    static constexpr int IB = sizeof(R) == 4 ? 16 : 8;
+    static constexpr int IB = sizeof(R) == 4 ? 16 : FMMFFT_NEAR_IB_D;
     static constexpr int TILE = sizeof(R) == 4 ? kTileF : kTileD;
     size_t QP() const { return (size_t)p->Q * p->P; }
     int nb_at(int lev) const { return (int)((1LL << lev) / p->G); }
@@ -852,6 +859,24 @@ struct Exec {
                     else
                         launch_pdl(k_s2t_tc<1>, grid, S2TC_THREADS, s2tc_smem_bytes(), side(), (const C*)rb.Sp, (const C*)rb.haloL,
                                    (const C*)rb.haloR, (float*)rb.Tn, (const float*)p->toep, p->P, p->nb, p->G, tpc);
+                    LAUNCH_CHECK();
+                }
+                if ((st = mark_on(p->ev_s2t[1], side()))) return st;
+                CUDA_TRY(cudaEventRecord(p->join, side()));
+                return FMMFFT_SUCCESS;
+            }
+        }
+        if constexpr (sizeof(R) == 8) {
+            if (p->M_L == 64 && p->nb % 32 == 0) {         // FP64 tensor pipe (mma.sync f64), k_s2t_dmma
+                constexpr int NB = 32;
+                for (RankBufs& rb : p->ranks) {
+                    const C* S = in[p->virt ? rb.g : 0];
+                    const size_t box = (size_t)p->M_L * p->P;
+                    const C* hl = p->G == 1 ? S + (size_t)(p->nb - 1) * box : (const C*)rb.haloL;
+                    const C* hr = p->G == 1 ? S : (const C*)rb.haloR;
+                    launch_pdl(k_s2t_dmma<NB>, dim3((unsigned)p->P, (unsigned)(p->nb / NB)), NB * 4, 0, side(),
+                               (const double2*)S, (const double2*)hl, (const double2*)hr, (double2*)rb.Tn,
+                               (const double*)p->s2t, p->s2t_chunk, p->PCn, p->P, p->nb);
                     LAUNCH_CHECK();
                 }
                 if ((st = mark_on(p->ev_s2t[1], side()))) return st;

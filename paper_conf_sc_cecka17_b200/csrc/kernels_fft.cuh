@@ -837,8 +837,11 @@ k_c2r_pre(const C2<R>* __restrict__ X, C2<R>* __restrict__ Zc, long long H) {
 // applies POST, runs the P-point DFT in registers (radix 2/4/8/16, 32 = 2 x 16) and stores
 // W[k2][b M_L + m] for every k2 (coalesced over m). CTA = NBX consecutive boxes x M_L threads.
 // ---------------------------------------------------------------------------------------------
+#ifndef FMMFFT_PPR_MINB
+#define FMMFFT_PPR_MINB 1            // k_post_pfft_r CTAs per SM the register budget is sized for
+#endif
 template <typename R, int LP, int QT>
-__global__ void __launch_bounds__(256)
+__global__ void __launch_bounds__(256, FMMFFT_PPR_MINB)
 k_post_pfft_r(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2<R>* __restrict__ r,
               const C2<R>* __restrict__ rho, const R* __restrict__ s2m, C2<R>* __restrict__ W, int lML, int Mg, int pmaj) {
     pdl_trigger();
