@@ -588,6 +588,10 @@ static fmmfft_status_t init_kernel_attrs() {
         set((const void*)k_down_narrow<R, 8>);
         set((const void*)k_down_narrow<R, 16>);
         set((const void*)k_down_narrow<R, 24>);
+        if constexpr (sizeof(R) == 8) {
+            set((const void*)k_m2l_dmma<8>); set((const void*)k_m2l_dmma<16>); set((const void*)k_m2l_dmma<24>);
+            set((const void*)k_m2m_dmma<8>); set((const void*)k_m2m_dmma<16>); set((const void*)k_m2m_dmma<24>);
+        }
         set((const void*)k_m2l_lvl<R, 8>);
         set((const void*)k_m2m_lvl<R, 8>);
         set((const void*)k_m2m_lvl<R, 16>);
@@ -942,8 +946,12 @@ struct Exec {
                 const size_t smem = m2m_lvl_smem<R, QV>();
                 const int per_sm = std::max(1, std::min(2, (int)((size_t)(optin + 1024) / (smem + 1024))));
                 const int nseg = (int)std::max(1LL, std::min<long long>(ntiles, (148LL * per_sm + nsub - 1) / nsub));
-                launch_pdl(k_m2m_lvl<R, QV>, dim3((unsigned)nseg, (unsigned)nsub), lvl_threads<R, QV>(), smem, s, src, o,
-                           (const R*)p->m2m, p->P, ntiles);
+                if constexpr (sizeof(R) == 8)                // FP64 tensor pipe
+                    launch_pdl(k_m2m_dmma<QV>, dim3((unsigned)nseg, (unsigned)nsub), 256, smem, s, (const C*)src, o,
+                               (const double*)p->m2m, p->P, ntiles);
+                else
+                    launch_pdl(k_m2m_lvl<R, QV>, dim3((unsigned)nseg, (unsigned)nsub), lvl_threads<R, QV>(), smem, s, src, o,
+                               (const R*)p->m2m, p->P, ntiles);
             });
             LAUNCH_CHECK();
             src = o;
@@ -1268,8 +1276,11 @@ struct Exec {
                     const int per_sm = std::max(1, std::min(2, (int)((size_t)(optin + 1024) / (smem + 1024))));
                     const int target = 148 * per_sm;
                     const int nseg = (int)std::max(1LL, std::min<long long>(la.ntiles, (target + nsub - 1) / nsub));
-                    launch_pdl(k_m2l_lvl<R, QV>, dim3((unsigned)nseg, (unsigned)nsub), lvl_threads<R, QV>(), smem, s, la,
-                               (const R*)p->m2m, p->P);
+                    if constexpr (sizeof(R) == 8)            // FP64 tensor pipe
+                        launch_pdl(k_m2l_dmma<QV>, dim3((unsigned)nseg, (unsigned)nsub), 256, smem, s, la, (const double*)p->m2m, p->P);
+                    else
+                        launch_pdl(k_m2l_lvl<R, QV>, dim3((unsigned)nseg, (unsigned)nsub), lvl_threads<R, QV>(), smem, s, la,
+                                   (const R*)p->m2m, p->P);
                 });
                 if (!ok) return fail(FMMFFT_UNSUPPORTED, "k_m2l_lvl: Q=%d", p->Q);
                 LAUNCH_CHECK();

@@ -70,7 +70,10 @@ __device__ __forceinline__ double2 twiddle_pow2(double, int e, int ls) {
 // 2^LLEN + 1 (padding against bank conflicts). For each butterfly j < len/E, k = j mod Ns:
 //   v_t = x[j + t len/E] w_{Ns E}^{k t};  v = DFT_E(v);  y[(j - k) E + k + t Ns] = v_t.
 // In place: each thread keeps its 8/E butterflies in registers across a barrier.
-// tw[u] = w_len^u, u < len.
+// tw[u] = w_len^u, u < len. Lanes run over COLUMNS (consecutive columns, same butterfly j): the
+// Stockham write y[(j - k) E + k + t Ns] then lands on a stride of the column pitch (P + 1
+// complex: at most 2-way bank conflicts) instead of a stride of E elements within one column
+// (up to 16-way for E = 8), and the warp's twiddle is a broadcast.
 template <int E, int LLEN, int LNS, typename C>
 __device__ __forceinline__ void stockham_stage(C* tile, int ncols, const C* tw) {
     constexpr int NB = 8 / E;
@@ -86,7 +89,7 @@ __device__ __forceinline__ void stockham_stage(C* tile, int ncols, const C* tw) 
     for (int k = 0; k < NB; ++k) {
         const int bf = tid + k * nthr;
         if (bf < total) {
-            const int col = bf >> LPER, j = bf & ((1 << LPER) - 1);
+            const int col = bf & (ncols - 1), j = bf / ncols;
             const C* x = tile + col * LD + j;
 #pragma unroll
             for (int t = 0; t < E; ++t) v[k][t] = x[t << LPER];
@@ -103,7 +106,7 @@ __device__ __forceinline__ void stockham_stage(C* tile, int ncols, const C* tw) 
     for (int k = 0; k < NB; ++k) {
         const int bf = tid + k * nthr;
         if (bf < total) {
-            const int col = bf >> LPER, j = bf & ((1 << LPER) - 1), kk = j & (NS - 1);
+            const int col = bf & (ncols - 1), j = bf / ncols, kk = j & (NS - 1);
             C* y = tile + col * LD + ((j - kk) << LE) + kk;
 #pragma unroll
             for (int t = 0; t < E; ++t) y[t << LNS] = v[k][t];
