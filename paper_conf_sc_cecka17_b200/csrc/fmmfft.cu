@@ -413,7 +413,15 @@ static fmmfft_status_t build_tables(fmmfft_plan_s* p) {
     return FMMFFT_SUCCESS;
 }
 
-static constexpr int kTileF = 8192, kTileD = 4096;   // shared FFT tile (elements)
+#ifndef FMMFFT_TILE_F
+#define FMMFFT_TILE_F 2048
+#endif
+#ifndef FMMFFT_TILE_D
+#define FMMFFT_TILE_D 2048
+#endif
+// shared FFT tile (elements) of k_post_pfft / k_fft_pass: 2048 = 256 threads per CTA, several CTAs
+// per SM overlap their load / compute / store phases (measured: 8192 -> 4096 -> 2048 = 98 -> 65 -> 59 us at P = 128)
+static constexpr int kTileF = FMMFFT_TILE_F, kTileD = FMMFFT_TILE_D;
 template <typename R> static constexpr int kRowFftMax = sizeof(R) == 4 ? 14 : 13;   // k_fft_row: whole row in smem
 // four-step passes: largest pass length (log2) and columns (rows) per CTA for a pass of 2^l points
 template <typename R> __host__ __device__ constexpr int fs_max() { return sizeof(R) == 4 ? 11 : 10; }
