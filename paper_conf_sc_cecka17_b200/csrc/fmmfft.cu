@@ -536,6 +536,10 @@ static void destroy_plan(fmmfft_plan_s* p) {
 #define FMMFFT_NEAR_IB_D 8           // complex128 k_near_up: outputs per thread (register block)
 #endif
 
+#ifndef FMMFFT_NARROW_FORCE
+#define FMMFFT_NARROW_FORCE 0        // 1: narrow kernels for the top of every tree, per-level kernels below
+#endif
+
 // Raise every kernel's dynamic shared memory cap once per device (function attributes are
 // per device; not legal during capture). Called with the plan's device current.
 template <typename R>
@@ -945,7 +949,7 @@ struct Exec {
         int optin = 0;
         CUDA_TRY(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, p->device));
         while (lvl_ok && cur > to && (nbc >> 1) >= 2 * lvl_nt<R, 16>() &&
-               (long long)((nbc >> 1) / lvl_nt<R, 16>()) * (p->P / PCl) >= 148) {
+               ((long long)((nbc >> 1) / lvl_nt<R, 16>()) * (p->P / PCl) >= 148 || (FMMFFT_NARROW_FORCE && narrow_ok() && !narrow_up_fits(nbc)))) {
             C* o = (C*)outs(cur - 1);
             const int nsub = p->P / PCl;
             dispatch<8, 16, 24>(p->Q, [&](auto qv) {
@@ -1186,7 +1190,7 @@ struct Exec {
             }
             constexpr int PCl = lvl_pc<R>();
             const bool lvl_usable = p->PCd % PCl == 0 && p->P % PCl == 0;
-            if (lnar > p->B && lnar == lnew - 1 && (lnar == p->L || lvl_usable)) {   // every narrow level
+            if (lnar > p->B && (lnar == lnew - 1 || FMMFFT_NARROW_FORCE) && (lnar == p->L || lvl_usable)) {
                 for (RankBufs& rb : p->ranks) {
                     const long long g = grank(rb);
                     NarrowArgs na{};
@@ -1194,7 +1198,10 @@ struct Exec {
                         const TreeLevel tl = level_io(rb, lev, g);
                         NarrowLevel& nl = na.lev[lev];
                         nl.src = tl.src; nl.src_base = tl.src_base; nl.src_mod = tl.src_mod;
-                        nl.tab = p->m2l_pmaj[lev]; nl.out = tl.out; nl.out_base = tl.out_base;
+                        nl.tab = p->m2l_pmaj[lev]; nl.out_base = tl.out_base;
+                        // only the last level leaves the chip (the per-level kernels' parent / the leaf
+                        // L^L); debug plans keep every level for the stage tests
+                        nl.out = (lev == lnar || (p->flags & FMMFFT_FLAG_DEBUG)) ? tl.out : nullptr;
                         const auto ft = narrow_targets(g, lev);
                         nl.f = ft.first; nl.n = ft.second;
                     }
@@ -1303,7 +1310,7 @@ struct Exec {
         if (p->P <= 32 && p->P >= 2 && (p->Q == 8 || p->Q == 16 || p->Q == 24) && p->M_L <= 256) {
             const int nbx = std::max(1, std::min(p->nb, 256 / p->M_L));
             if (p->nb % nbx == 0) {
-                const size_t smem = ((size_t)nbx * p->Q * p->P + 2 * p->P + 16) * sizeof(C);
+                const size_t smem = ((size_t)nbx * p->Q * p->P + 2 * p->P + 16) * sizeof(C) + (size_t)p->Q * p->M_L * sizeof(R);
                 for (RankBufs& rb : p->ranks) {
                     bool ok = dispatch<1, 2, 3, 4, 5>(ilog2(p->P), [&](auto lp) {
                         constexpr int LP = decltype(lp)::value;
@@ -1321,7 +1328,7 @@ struct Exec {
         }
         // m sub-tile per CTA: the whole P-point FFT tile, split further (down to 16) while that
         // leaves fewer than ~4 CTAs per SM (small N: latency-bound, more CTAs in flight)
-        int MS = std::min(p->M_L, std::max(1, TILE / p->P));
+        int MS = std::min(p->M_L, std::max(8, TILE / p->P));     // >= 8: the L2T phase owns 8 m per thread
         while (MS > 16 && (long long)p->nb * (p->M_L / MS) < 4 * 148) MS /= 2;
         const int threads = std::min(sizeof(R) == 4 ? 1024 : 512, std::max(32, MS * p->P / 8));
         size_t smem = (size_t)MS * (p->P + 1) * sizeof(C) + (size_t)p->P * sizeof(C) + (size_t)p->Q * MS * sizeof(R);

@@ -841,7 +841,7 @@ k_c2r_pre(const C2<R>* __restrict__ X, C2<R>* __restrict__ Zc, long long H) {
 // W[k2][b M_L + m] for every k2 (coalesced over m). CTA = NBX consecutive boxes x M_L threads.
 // ---------------------------------------------------------------------------------------------
 #ifndef FMMFFT_PPR_MINB
-#define FMMFFT_PPR_MINB 1            // k_post_pfft_r CTAs per SM the register budget is sized for
+#define FMMFFT_PPR_MINB 3            // k_post_pfft_r CTAs per SM the register budget is sized for
 #endif
 template <typename R, int LP, int QT>
 __global__ void __launch_bounds__(256, FMMFFT_PPR_MINB)
@@ -857,11 +857,10 @@ k_post_pfft_r(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const 
     C* rr = Lsm + nbx * Q * P;                                     // [P] r_p
     C* rh = rr + P;                                                // [P] rho_p
     C* tw32 = rh + P;                                              // [16] w_32^k
+    R* wsm = reinterpret_cast<R*>(tw32 + 16);                      // [Q][M_L] L2T_{mq} = S2M_{qm}
     const int tid = threadIdx.x, bx = tid >> lML, m = tid & (M_L - 1);
     const int b = blockIdx.x * nbx + bx;
-    R w[Q];                                                        // L2T_{mq} = S2M_{qm}
-#pragma unroll
-    for (int q = 0; q < Q; ++q) w[q] = __ldg(s2m + (size_t)q * M_L + m);
+    for (int idx = tid; idx < Q * M_L; idx += blockDim.x) cp_async_elem(wsm + idx, s2m + idx);
     if (tid < 16) tw32[tid] = twiddle_pow2(R(0), tid, 5);
     pdl_wait();                                                   // T_near / L^L / r from the FMM stages
     {
@@ -888,32 +887,20 @@ k_post_pfft_r(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const 
     }
     cp_async_wait_all();
     __syncthreads();
+    // L2T accumulated straight into the column (q outer: one L2T coefficient register, the L^L
+    // row of q a broadcast), then POST; p = 0 is the identity (C_0 = I, R1)
     const C* Lb = Lsm + bx * Q * P;
+#pragma unroll 4
+    for (int q = 0; q < Q; ++q) {
+        const R wq = wsm[q * M_L + m];
 #pragma unroll
-    for (int p = 0; p < P; p += 2) {
-        C a0 = zero<C>(), a1 = zero<C>();
+        for (int p = 1; p < P; ++p) rfma(v[p], wq, pmaj ? Lb[p * Q + q] : Lb[q * P + p]);
+    }
 #pragma unroll
-        for (int q = 0; q < Q; ++q) {
-            C l0, l1;
-            if (pmaj) {                                            // broadcast loads, [p][q]
-                l0 = Lb[p * Q + q]; l1 = Lb[(p + 1) * Q + q];
-            } else if constexpr (sizeof(R) == 4) {
-                const float4 l = *reinterpret_cast<const float4*>(Lb + q * P + p);
-                l0 = make_float2(l.x, l.y); l1 = make_float2(l.z, l.w);
-            } else {
-                l0 = Lb[q * P + p]; l1 = Lb[q * P + p + 1];
-            }
-            rfma(a0, w[q], l0);
-            rfma(a1, w[q], l1);
-        }
-        if (p > 0) {                                               // C_0 = I (R1)
-            C t = cadd(v[p], a0);
-            t.x -= rr[p].y; t.y += rr[p].x;                        // + i r_p
-            v[p] = cmul(rh[p], t);
-        }
-        C t = cadd(v[p + 1], a1);
-        t.x -= rr[p + 1].y; t.y += rr[p + 1].x;
-        v[p + 1] = cmul(rh[p + 1], t);
+    for (int p = 1; p < P; ++p) {
+        C t = v[p];
+        t.x -= rr[p].y; t.y += rr[p].x;                            // + i r_p
+        v[p] = cmul(rh[p], t);
     }
     // P-point DFT over p, natural order
     if constexpr (P <= 16) {
