@@ -101,7 +101,14 @@ typedef enum {
                                    X_0 and X_{N/2} are ignored): one elementwise pass (k_c2r_pre)
                                    builds the length-N/2 spectrum of z_j = x_{2j} + i x_{2j+1},
                                    then the inverse complex plan writes z = the N reals in place.
-                                   G = 1 only, not with VIRTUAL (else FMMFFT_UNSUPPORTED).
+                                   G > 1: x block-distributed (rank g holds reals
+                                   [g N/G, (g+1) N/G)); rank g's out holds X_k for k in
+                                   [g N/(2G), (g+1) N/(2G)) plus one slot, written only by rank
+                                   G-1 with X_{N/2} (so every rank's out is N/(2G) + 1 complex;
+                                   VIRTUAL plans: one array X_0..X_{N/2}); the inverse takes the
+                                   same distribution. One extra exchange per execute: rank g
+                                   receives rank G-1-g's block and one element (the pairing of
+                                   k with N/2 - k crosses ranks).
                                    fmmfft_get_info reports the real N; M, L, ... describe the
                                    complex plan. */
 
@@ -186,6 +193,8 @@ typedef struct {
 
 #define FMMFFT_VARIANT_TREE_FUSED 1u  /* far field as one per-FMM kernel (G = 1, tree fits smem) */
 #define FMMFFT_VARIANT_S2T_TC     2u  /* near field on tcgen05 tensor cores (3xTF32)             */
+#define FMMFFT_VARIANT_S2T_FFT  128u  /* near field as a fast convolution: per-box DFT_128, 3
+                                         kernel spectra, inverse DFT_128 (k_s2t_fft, NEXT-4)       */
 #define FMMFFT_VARIANT_ROW_FFT1   4u  /* M-point FFTs as one single-pass kernel per row        */
 #define FMMFFT_VARIANT_FOURSTEP   8u  /* long rows: column pass(es) + transposing row pass     */
 #define FMMFFT_VARIANT_DOWN_LVL  32u  /* wide levels on the per-level M2M / M2L kernels        */

@@ -153,17 +153,15 @@ def fmmfft_rank(x_local: np.ndarray, N: int, P: int, B: int, Q: int, M_L: int,
     return Y.reshape(Pl * M)
 
 
-def fmmfft_virtual(x: np.ndarray, P: int, B: int, Q: int, M_L: int = 64, G: int = 2) -> np.ndarray:
-    """Run G ranks in threads on the blocks of x; return the concatenated output blocks."""
-    x = np.asarray(x, dtype=np.complex128)
-    N = len(x)
+def _run_threads(G: int, fn):
+    """fn(g, comm) on G threads sharing one ThreadGroup; returns the G results in rank order."""
     comm = ThreadGroup(G)
     outs = [None] * G
     errs = []
 
     def run(g):
         try:
-            outs[g] = fmmfft_rank(x[g * N // G:(g + 1) * N // G], N, P, B, Q, M_L, g, G, comm)
+            outs[g] = fn(g, comm)
         except BaseException as e:  # noqa: BLE001 - surface worker errors to the caller
             errs.append(e)
             comm._bar.abort()
@@ -175,4 +173,98 @@ def fmmfft_virtual(x: np.ndarray, P: int, B: int, Q: int, M_L: int = 64, G: int 
         t.join()
     if errs:
         raise errs[0]
-    return np.concatenate(outs)
+    return outs
+
+
+def fmmfft_virtual(x: np.ndarray, P: int, B: int, Q: int, M_L: int = 64, G: int = 2) -> np.ndarray:
+    """Run G ranks in threads on the blocks of x; return the concatenated output blocks."""
+    x = np.asarray(x, dtype=np.complex128)
+    N = len(x)
+    return np.concatenate(_run_threads(G, lambda g, comm: fmmfft_rank(x[g * N // G:(g + 1) * N // G], N, P, B, Q,
+                                                                       M_L, g, G, comm)))
+
+
+# --------------------------------------------------------------------------------------------
+# Real input at G ranks (reading R18, SURVEY §8(f) NEXT-1): N reals block-distributed, packed as
+# z_j = x_{2j} + i x_{2j+1} (rank g's z block is its own reals), the distributed complex FMM-FFT
+# of length H = N/2, then X_k = E_k + w_N^k O_k with E_k = (Z_k + conj Z_{H-k})/2,
+# O_k = -i (Z_k - conj Z_{H-k})/2. Z_{H-k} for rank g's k lives on rank G-1-g (and one element,
+# A[(G-g) H/G], on rank (G-g) mod G): the mirror exchange below. Output: rank g holds X_k for
+# k in [g H/G, (g+1) H/G); the last rank also X_H.
+# --------------------------------------------------------------------------------------------
+def mirror_exchange(A_local: np.ndarray, extra_H, rank: int, G: int, comm, c2r: bool):
+    """Rank g receives rank G-1-g's block and the element A[(G-g) H/G] (A[H] = Z[0] for the
+    forward — rank 0's first element; = X_H for the inverse — rank G-1's extra value extra_H)."""
+    nl = len(A_local)
+    chunks = [np.zeros(nl + 2, dtype=np.complex128) for _ in range(G)]
+    chunks[G - 1 - rank][:nl] = A_local
+    if not c2r:
+        chunks[(G - rank) % G][nl] = A_local[0]
+    else:
+        if rank > 0:
+            chunks[G - rank][nl] = A_local[0]
+        if rank == G - 1:
+            chunks[0][nl + 1] = extra_H
+    got = comm.alltoall(rank, chunks)
+    mir = np.asarray(got[G - 1 - rank][:nl])
+    if not c2r:
+        xtra = got[(G - rank) % G][nl]
+    else:
+        xtra = got[G - 1][nl + 1] if rank == 0 else got[G - rank][nl]
+    return mir, xtra
+
+
+def rdft_rank(x_local: np.ndarray, N: int, P: int, B: int, Q: int, M_L: int, rank: int, G: int, comm) -> np.ndarray:
+    """Rank g's X_k, k in its block (+ X_{N/2} on the last rank), of N block-distributed reals."""
+    H = N // 2
+    nl = H // G
+    x_local = np.asarray(x_local, dtype=np.float64)
+    z = x_local[0::2] + 1j * x_local[1::2]
+    Z = fmmfft_rank(z, H, P, B, Q, M_L, rank, G, comm)
+    mir, xtra = mirror_exchange(Z, None, rank, G, comm, c2r=False)
+    j = np.arange(nl)
+    zb = np.concatenate([[xtra], mir[nl - j[1:]]])                     # Z_{H-k}
+    k = rank * nl + j
+    E = (Z + np.conj(zb)) / 2
+    Od = -1j * (Z - np.conj(zb)) / 2
+    X = E + np.exp(-2j * np.pi * k / N) * Od
+    if rank == G - 1:                                                  # X_H = E_0 - O_0 from Z_0
+        X = np.concatenate([X, [mir[0].real - mir[0].imag]])
+    return X
+
+
+def irdft_rank(X_local: np.ndarray, N: int, P: int, B: int, Q: int, M_L: int, rank: int, G: int, comm) -> np.ndarray:
+    """The inverse: rank g's N/G reals from its X block (the last rank's block ends with X_{N/2});
+    the imaginary parts of X_0 and X_{N/2} are ignored (a real signal's are zero)."""
+    H = N // 2
+    nl = H // G
+    X_local = np.asarray(X_local, dtype=np.complex128)
+    a = X_local[:nl].copy()
+    mir, xtra = mirror_exchange(a, X_local[nl] if rank == G - 1 else None, rank, G, comm, c2r=True)
+    j = np.arange(nl)
+    xb = np.concatenate([[xtra], mir[nl - j[1:]]])                     # X_{H-k}
+    k = rank * nl + j
+    if rank == 0:
+        a[0], xb[0] = a[0].real, xb[0].real
+    E = (a + np.conj(xb)) / 2
+    Od = np.exp(2j * np.pi * k / N) * (a - np.conj(xb)) / 2
+    Z = E + 1j * Od                                                    # DFT_H of z_j = x_{2j} + i x_{2j+1}
+    z = np.conj(fmmfft_rank(np.conj(Z), H, P, B, Q, M_L, rank, G, comm)) / H
+    x = np.empty(2 * nl)
+    x[0::2], x[1::2] = z.real, z.imag
+    return x
+
+
+def rdft_virtual(x: np.ndarray, P: int, B: int, Q: int, M_L: int = 64, G: int = 2) -> np.ndarray:
+    x = np.asarray(x, dtype=np.float64)
+    N = len(x)
+    return np.concatenate(_run_threads(G, lambda g, comm: rdft_rank(x[g * N // G:(g + 1) * N // G], N, P, B, Q, M_L,
+                                                                    g, G, comm)))
+
+
+def irdft_virtual(X: np.ndarray, P: int, B: int, Q: int, M_L: int = 64, G: int = 2) -> np.ndarray:
+    X = np.asarray(X, dtype=np.complex128)
+    N = 2 * (len(X) - 1)
+    nl = N // 2 // G
+    blk = lambda g: X[g * nl:(g + 1) * nl + (1 if g == G - 1 else 0)]   # noqa: E731
+    return np.concatenate(_run_threads(G, lambda g, comm: irdft_rank(blk(g), N, P, B, Q, M_L, g, G, comm)))

@@ -38,6 +38,7 @@
 #include "kernels_fft.cuh"
 #include "kernels_fmm.cuh"
 #include "kernel_s2t_tc.cuh"
+#include "kernel_s2t_fft.cuh"
 #include "nccl_loader.hpp"
 
 namespace fmmfft {
@@ -201,6 +202,8 @@ struct RankBufs {
     void* dc = nullptr;      // [P/G] the k1 = 0 outputs of this rank's M-FFT rows (k_dc_bins, R19)
     void* cin = nullptr;     // conj(in) (inverse plans)
     void* rz = nullptr;      // Z = F_{N/2} z (real-input plans, FMMFFT_FLAG_REAL)
+    void* mir = nullptr;     // real plans, G > 1: the mirror block (rank G-1-g's Z or X block)
+    void* xtra = nullptr;    //   and the one element A[(G-g) N/(2G)] (mirror exchange)
     void* din = nullptr;     // execute_host staging
     void* dout = nullptr;
     std::vector<void*> Mpad, Lloc, Mfull, Lfull;   // indexed by level
@@ -242,6 +245,9 @@ struct fmmfft_plan_s {
     bool pmaj = false;               // M^L / L^L p-major [p][b][q] between k_s2m, k_tree_pc and post_pfft
     bool direct = false;             // FMMFFT_FLAG_DIRECT: plain four-step FFT of length N, no FMM
     bool s2t_tc = false;             // S2T on tcgen05 (k_s2t_tc): complex64, M_L = 64, nb % 128 == 0
+    bool s2t_fft = false;            // S2T as a fast convolution (k_s2t_fft, NEXT-4): M_L = 64, nb % 32 == 0
+    bool s2t_dmma = false;           // complex128 S2T direct sum on the FP64 tensor pipe (k_s2t_dmma)
+    void* s2tf_h = nullptr;          // its kernel spectra H_s = DFT_128(h_s) / 128, [p][s][cc][k1][t']
     void* toep = nullptr;            // its Toeplitz hi/lo operand table
     bool row_fft1 = false;           // M-point FFTs in one pass per row (k_fft_row), M fits smem
     void* twM = nullptr;             // its twiddles w_M^u, u < M/16
@@ -393,6 +399,33 @@ static fmmfft_status_t build_tables(fmmfft_plan_s* p) {
         fmmfft_status_t st2 = dalloc(p, &p->toep, tb.size() * sizeof(float));
         if (st2) return st2;
         CUDA_TRY(cudaMemcpy(p->toep, tb.data(), tb.size() * sizeof(float), cudaMemcpyHostToDevice));
+    }
+    // fast-convolution S2T (kernel_s2t_fft.cuh): h_s[n mod 128] = S2T_{p, 64 s - n} for
+    // n in [-63, 63] (s = -1, 0, 1), h_s[64] = 0; H_s[f] = sum_n h_s[n] w_128^{f n} / 128 (float64,
+    // exact angle reduction f n mod 128), stored [p][s][cc][k1][t'] with f = 2 t' + cc + 16 k1
+    if (p->s2t_fft) {
+        std::vector<double> cs(128), sn(128);
+        for (int k = 0; k < 128; ++k) { cs[k] = std::cos(2 * M_PI * k / 128.0); sn[k] = -std::sin(2 * M_PI * k / 128.0); }
+        std::vector<double> H((size_t)P * S2TF_H_PER_P * 2, 0.0);
+        for (int pp = 0; pp < P; ++pp)
+            for (int s = -1; s <= 1; ++s) {
+                double h[128];
+                for (int n = 0; n < 128; ++n) {
+                    const int lag = n <= 63 ? n : n - 128;          // n = 64: unused slot
+                    const long long k = 64LL * s - lag;
+                    h[n] = n == 64 ? 0.0
+                                   : (pp == 0 ? (k == 0 ? 1.0 : 0.0) : cotpi((double)(pp + (long long)P * k) / (double)N));
+                }
+                for (int f = 0; f < 128; ++f) {
+                    double re = 0, im = 0;
+                    for (int n = 0; n < 128; ++n) { re += h[n] * cs[(f * n) & 127]; im += h[n] * sn[(f * n) & 127]; }
+                    const int k2 = f & 15, k1 = f >> 4, tt = k2 >> 1, cc = k2 & 1;
+                    const size_t e = (size_t)pp * S2TF_H_PER_P + (size_t)(s + 1) * 128 + (cc * 8 + k1) * 8 + tt;
+                    H[2 * e] = re / 128.0;
+                    H[2 * e + 1] = im / 128.0;
+                }
+            }
+        if ((st = upload<R>(p, &p->s2tf_h, H))) return st;
     }
     // rho_p = exp(-i pi p/P) sin(pi p/P) / M, interleaved complex; rho_0 unused
     std::vector<double> rho(2 * (size_t)P);
@@ -587,6 +620,7 @@ static fmmfft_status_t init_kernel_attrs() {
             set((const void*)k_tree_pc<8, 512, 2>);
         }
         if constexpr (sizeof(R) == 4) { set((const void*)k_s2t_tc<1>); set((const void*)k_s2t_tc<2>); }
+        set((const void*)k_s2t_fft<R>);
         set((const void*)k_base_sg<R, 4, sizeof(R) == 4 ? 8 : 4, 4>);
         for (int lp = 1; lp <= 5; ++lp)
             dispatch<1, 2, 3, 4, 5>(lp, [&](auto v) {
@@ -742,6 +776,26 @@ struct Exec {
         return v;
     }
 
+    // real plans, G > 1: the mirror exchange. Output k of rank g needs A[H - k] (H = N/2, A = Z
+    // for the forward, A = X for the inverse): for k in g's block those are rank G-1-g's block
+    // (reversed, minus its first element) and the one element A[(G-g) H/G] — rank (G-g) mod G's
+    // first (R2C: A[H] = Z[0], rank 0's own), or for C2R at g = 0 X_H, rank G-1's extra slot
+    std::vector<P2P> sched_mirror(const RankBufs& rb, const C* own, bool c2r) const {
+        const int G = p->G, g = grank(rb);
+        const size_t nl = (size_t)(p->N / G);
+        C* a = const_cast<C*>(own);
+        std::vector<P2P> v;
+        v.push_back({true, G - 1 - g, a, nl});                          // mirror block first
+        if (!c2r) v.push_back({true, (G - g) % G, a, 1});
+        else {
+            if (g == G - 1) v.push_back({true, 0, a + nl, 1});           // X_H -> rank 0
+            if (g > 0) v.push_back({true, G - g, a, 1});
+        }
+        v.push_back({false, G - 1 - g, rb.mir, nl});
+        v.push_back({false, c2r ? (g == 0 ? G - 1 : G - g) : (G - g) % G, rb.xtra, 1});
+        return v;
+    }
+
     // issue one exchange on stream st: NCCL group (one process per GPU), or every virtual rank's
     // list matched send-to-receive and executed as device copies (or NCCL self send / receive on
     // a 1-rank communicator, FMMFFT_FLAG_VIRTUAL_NCCL)
@@ -858,6 +912,23 @@ struct Exec {
         CUDA_TRY(cudaEventRecord(p->fork2, s));
         CUDA_TRY(cudaStreamWaitEvent(side(), p->fork2, 0));
         if ((st = mark_on(p->ev_s2t[0], side()))) return st;
+        if (p->s2t_fft) {                                      // fast convolution (k_s2t_fft, NEXT-4)
+            const long long nchunk = p->nb / S2TF_CHUNK;
+            // chunks per CTA: >= ~4 waves of 148 SMs x 4 CTAs, at most 16 (prologue = 1/cpc of a chunk)
+            const int cpc = (int)std::max<long long>(1, std::min<long long>(16, nchunk * p->P / (148 * 16)));
+            for (RankBufs& rb : p->ranks) {
+                const C* S = in[p->virt ? rb.g : 0];
+                const size_t box = (size_t)p->M_L * p->P;
+                const C* hl = p->G == 1 ? S + (size_t)(p->nb - 1) * box : (const C*)rb.haloL;
+                const C* hr = p->G == 1 ? S : (const C*)rb.haloR;
+                launch_pdl(k_s2t_fft<R>, dim3((unsigned)p->P, (unsigned)((nchunk + cpc - 1) / cpc)), S2TF_THREADS,
+                           s2tf_smem_bytes<R>(), side(), S, hl, hr, (R*)rb.Tn, (const C*)p->s2tf_h, p->P, p->nb, cpc);
+                LAUNCH_CHECK();
+            }
+            if ((st = mark_on(p->ev_s2t[1], side()))) return st;
+            CUDA_TRY(cudaEventRecord(p->join, side()));
+            return FMMFFT_SUCCESS;
+        }
         if constexpr (sizeof(R) == 4) {
             if (p->s2t_tc) {                                   // tensor cores (tcgen05, 3xTF32)
                 const int ntile = p->nb / S2TC_BOXES;
@@ -883,7 +954,7 @@ struct Exec {
             }
         }
         if constexpr (sizeof(R) == 8) {
-            if (p->M_L == 64 && p->nb % 32 == 0) {         // FP64 tensor pipe (mma.sync f64), k_s2t_dmma
+            if (p->s2t_dmma) {                                 // FP64 tensor pipe (mma.sync f64), k_s2t_dmma
                 constexpr int NB = 32;
                 for (RankBufs& rb : p->ranks) {
                     const C* S = in[p->virt ? rb.g : 0];
@@ -1391,6 +1462,8 @@ struct Exec {
             int lblk = 62;
             if (p->G > 1 && src_override != in[0]) { in_row = p->Mg; lblk = ilog2(p->Mg); blk_stride = (p->P / p->G) * p->Mg; }
             if (p->fs_lr) {                      // four-step: column pass(es) + transposing row pass
+                // (running every pass of a group of rows back to back, so the group's intermediate
+                // stays in L2, measured slower at cfg3: 499 -> 524-538 us for groups of 4 / 2 rows)
                 const int npass = p->fs_lc2 ? 3 : 2;
                 C* a1out = npass == 3 ? dst : (C*)rb.tmp;
                 if ((st_ = col_pass(src, a1out, p->fs_lc1, lM, 0, in_row, lblk, blk_stride, rows))) return st_;
@@ -1498,19 +1571,42 @@ struct Exec {
         fmmfft_status_t st;
         if (p->real && p->inverse) {                    // C2R: conj(Z) -> forward -> conj / H = z
             const long long H = p->N;
-            C* Zc = (C*)p->ranks[0].cin;
-            const unsigned blocks = (unsigned)std::min<long long>((H / 2 + 256) / 256, 148LL * 8);
-            launch_pdl(k_c2r_pre<R>, blocks, 256, 0, s, in[0], Zc, H);
-            LAUNCH_CHECK();
-            in[0] = Zc;
+            if (p->G > 1 && (st = exchange([this](const RankBufs& rb) { return sched_mirror(rb, in[gidx(rb)], true); }, s)))
+                return st;
+            for (RankBufs& rb : p->ranks) {
+                const int g = gidx(rb);
+                C* Zc = (C*)rb.cin;
+                if (p->G == 1) {
+                    const unsigned blocks = (unsigned)std::min<long long>((H / 2 + 256) / 256, 148LL * 8);
+                    launch_pdl(k_c2r_pre<R>, blocks, 256, 0, s, in[g], Zc, H);
+                } else {
+                    const long long nl = H / p->G;
+                    const unsigned blocks = (unsigned)std::min<long long>((nl + 255) / 256, 148LL * 8);
+                    launch_pdl(k_c2r_pre_dist<R>, blocks, 256, 0, s, in[g], (const C*)rb.mir, (const C*)rb.xtra, Zc, H, nl,
+                               (long long)grank(rb) * nl);
+                }
+                LAUNCH_CHECK();
+                in[g] = Zc;
+            }
             if ((st = run_forward())) return st;
-            return conj_scale(out[0], out[0], R(1) / (R)H);
+            for (RankBufs& rb : p->ranks)
+                if ((st = conj_scale(out[gidx(rb)], out[gidx(rb)], R(1) / (R)H))) return st;
+            return FMMFFT_SUCCESS;
         }
         if (p->real) {                                  // z_j = x_{2j} + i x_{2j+1}: the input as is
-            C* X = out[0];
-            out[0] = (C*)p->ranks[0].rz;
+            std::vector<C*> X = out;
+            for (RankBufs& rb : p->ranks) out[gidx(rb)] = (C*)rb.rz;
             if ((st = run_forward())) return st;
-            return r2c_post(out[0], X);
+            if (p->G == 1) return r2c_post(out[0], X[0]);
+            if ((st = exchange([this](const RankBufs& rb) { return sched_mirror(rb, (const C*)rb.rz, false); }, s))) return st;
+            for (RankBufs& rb : p->ranks) {
+                const long long nl = p->N / p->G;
+                const unsigned blocks = (unsigned)std::min<long long>((nl + 255) / 256, 148LL * 8);
+                launch_pdl(k_r2c_post_dist<R>, blocks, 256, 0, s, (const C*)rb.rz, (const C*)rb.mir, (const C*)rb.xtra,
+                           X[gidx(rb)], p->N, nl, (long long)grank(rb) * nl, (int)(grank(rb) == p->G - 1));
+                LAUNCH_CHECK();
+            }
+            return FMMFFT_SUCCESS;
         }
         if (p->inverse)                                 // F^{-1} x = conj(F conj(x)) / N
             for (RankBufs& rb : p->ranks) {
@@ -1906,10 +2002,20 @@ static fmmfft_status_t plan_complex(fmmfft_plan_t* plan, long long N, int P, int
         // per FMM (k_tree_p)
         if (p->tree_p && precision == FMMFFT_C64 && (Q == 16 || Q == 8) && tree_pc_smem(p, 2) <= (size_t)optin) p->tree_cl = 2;
     }
-    // tensor-core S2T (k_s2t_tc, 3xTF32 on tcgen05) for complex64 with M_L = 64 and whole 128-box
-    // tiles per rank; FMMFFT_S2T=simt selects the FFMA2 kernel (k_near_up) instead
-    p->s2t_tc = precision == FMMFFT_C64 && M_L == 64 && (p->nb % S2TC_BOXES) == 0;
-    if (const char* e = getenv("FMMFFT_S2T")) p->s2t_tc = p->s2t_tc && e[0] == 't';
+    // S2T kernel: complex64 with M_L = 64 and whole 128-box tiles per rank -> tensor cores
+    // (k_s2t_tc, 3xTF32 on tcgen05); other M_L = 64 plans (32-box chunks) -> the fast convolution
+    // (k_s2t_fft, NEXT-4: measured 5.77 -> 5.15 ms against the FP64 tensor-pipe direct sum at cfg4,
+    // and 1.03 ms vs 1.85 ms for the FFMA2 kernel at cfg3's complex64 shape); else k_near_up.
+    // FMMFFT_S2T=tc | fft | dmma (complex128 direct sum on mma.sync f64) | simt (k_near_up) overrides
+    {
+        const bool tc_ok = precision == FMMFFT_C64 && M_L == 64 && (p->nb % S2TC_BOXES) == 0;
+        const bool fft_ok = M_L == 64 && (p->nb % S2TF_CHUNK) == 0;
+        const char* e = getenv("FMMFFT_S2T");
+        const char k = (e && *e) ? e[0] : 0;            // 0: the default choice
+        p->s2t_tc = tc_ok && (k == 't' || k == 0);
+        p->s2t_fft = fft_ok && (k == 'f' || ((k == 0 || k == 't') && !tc_ok));
+        p->s2t_dmma = precision == FMMFFT_C128 && M_L == 64 && (p->nb % 32) == 0 && !p->s2t_fft && k != 's';
+    }
     // the cluster far field gathers M^L and scatters L^L one FMM (one p) at a time: keep both
     // p-major so those are contiguous runs (debug plans keep [b][q][p] for the stage buffers)
     p->pmaj = p->tree_p && p->tree_cl > 1 && L > B && !(flags & FMMFFT_FLAG_DEBUG);
@@ -1999,23 +2105,25 @@ fmmfft_status_t fmmfft_autotune(long long N, int G, fmmfft_precision_t precision
 
 // FMMFFT_FLAG_REAL (SURVEY §8(f) NEXT-1, C = 1): N real inputs read as the complex vector
 // z_j = x_{2j} + i x_{2j+1} of length H = N/2, the complex plan of length H (FMM or DIRECT), then
-// k_r2c_post. G = 1 only; no INVERSE / VIRTUAL.
+// k_r2c_post; at G > 1 the mirror exchange (sched_mirror) + k_r2c_post_dist.
 fmmfft_status_t fmmfft_plan_ex(fmmfft_plan_t* plan, long long N, int P, int G, int B, int Q,
                                fmmfft_precision_t precision, int M_L, unsigned flags) {
     if (!(flags & FMMFFT_FLAG_REAL)) return plan_complex(plan, N, P, G, B, Q, precision, M_L, flags);
     if (!plan) return fail(FMMFFT_INVALID_VALUE, "plan is NULL");
     *plan = nullptr;
-    if (G != 1) return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_REAL: single GPU only (G = 1)");
-    if (flags & FMMFFT_FLAG_VIRTUAL) return fail(FMMFFT_UNSUPPORTED, "FMMFFT_FLAG_REAL: non-virtual plans only");
     if (N < 4 || (N & 1)) return fail(FMMFFT_INVALID_VALUE, "FMMFFT_FLAG_REAL: N must be even");
     fmmfft_status_t st = plan_complex(plan, N / 2, P, G, B, Q, precision, M_L, flags);
     if (st) return st;
     fmmfft_plan_s* p = *plan;
     p->real = true;
-    if ((st = dalloc(p, &p->ranks[0].rz, (size_t)(N / 2) * p->esz))) {
-        destroy_plan(p);
-        *plan = nullptr;
-        return st;
+    for (RankBufs& rb : p->ranks) {
+        const size_t nl = (size_t)(N / 2 / G);
+        if ((st = dalloc(p, &rb.rz, nl * p->esz)) ||
+            (G > 1 && ((st = dalloc(p, &rb.mir, nl * p->esz)) || (st = dalloc(p, &rb.xtra, p->esz))))) {
+            destroy_plan(p);
+            *plan = nullptr;
+            return st;
+        }
     }
     return FMMFFT_SUCCESS;
 }
@@ -2083,6 +2191,7 @@ fmmfft_status_t fmmfft_get_info(fmmfft_plan_t p, fmmfft_info_t* info) {
     info->L = p->L; info->precision = p->prec; info->M = p->M; info->level_gather = p->lg;
     info->n_stages = ST_COUNT + 1; info->workspace_bytes = p->ws_bytes; info->kernels_per_execute = p->kernels;
     info->variant = (p->tree_p ? FMMFFT_VARIANT_TREE_FUSED : 0u) | (p->s2t_tc ? FMMFFT_VARIANT_S2T_TC : 0u) |
+                    (p->s2t_fft ? FMMFFT_VARIANT_S2T_FFT : 0u) |
                     (p->row_fft1 ? FMMFFT_VARIANT_ROW_FFT1 : 0u) | (p->fs_lr ? FMMFFT_VARIANT_FOURSTEP : 0u) |
                     (!p->tree_p && !p->direct ? FMMFFT_VARIANT_DOWN_LVL : 0u) |
                     (p->pmaj ? FMMFFT_VARIANT_PMAJ : 0u);

@@ -794,6 +794,40 @@ k_r2c_post(const C2<R>* __restrict__ Z, C2<R>* __restrict__ X, long long H) {
     }
 }
 
+// k_r2c_post_dist: the same separation at G > 1 for rank g's block k = k0 + j, j < nl, with
+// Z_{H-k} from the mirror exchange (Zm = rank G-1-g's block, Z_{H-k} = Zm[nl - j] for j > 0,
+// zx = Z_{H-k0}); the last rank also writes X_H = Re Z_0 - Im Z_0 (Zm[0] = Z_0) at X[nl].
+template <typename R>
+__global__ void __launch_bounds__(256)
+k_r2c_post_dist(const C2<R>* __restrict__ Z, const C2<R>* __restrict__ Zm, const C2<R>* __restrict__ zx,
+                C2<R>* __restrict__ X, long long H, long long nl, long long k0, int last) {
+    pdl_trigger();
+    pdl_wait();
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    for (long long j = (long long)blockIdx.x * blockDim.x + threadIdx.x; j < nl; j += stride) {
+        const long long k = k0 + j;
+        const C2<R> a = Z[j];
+        const C2<R> zb = j == 0 ? zx[0] : Zm[nl - j];
+        const R Er = R(0.5) * (a.x + zb.x), Ei = R(0.5) * (a.y - zb.y);
+        const R Or = R(0.5) * (a.y + zb.y), Oi = R(-0.5) * (a.x - zb.x);
+        R wr, wi;                                                        // w_N^k = exp(-2 pi i k / 2H)
+        if constexpr (sizeof(R) == 4) {
+            float sn, cs;
+            sincospif(-(float)((double)k / (double)H), &sn, &cs);
+            wr = cs; wi = sn;
+        } else {
+            double sn, cs;
+            sincospi(-(double)k / (double)H, &sn, &cs);
+            wr = cs; wi = sn;
+        }
+        X[j] = C2<R>{Er + wr * Or - wi * Oi, Ei + wr * Oi + wi * Or};
+        if (last && j == 0) {
+            const C2<R> z0 = Zm[0];
+            X[nl] = C2<R>{z0.x - z0.y, R(0)};
+        }
+    }
+}
+
 // ---------------------------------------------------------------------------------------------
 // k_c2r_pre (FMMFFT_FLAG_REAL | FMMFFT_FLAG_INVERSE): from X_k, k = 0..H, of a real signal of
 // length N = 2H (X_{N-k} = conj(X_k)), with a = X_k, b = conj(X_{H-k}):
@@ -829,6 +863,38 @@ k_c2r_pre(const C2<R>* __restrict__ X, C2<R>* __restrict__ Zc, long long H) {
         Zc[k] = C2<R>{Er - Oi, -(Ei + Or)};
         // Z_{H-k} = conj(E) + i conj(O) = (Er + Oi) + i (Or - Ei); stored conjugated
         if (k != 0) Zc[H - k] = C2<R>{Er + Oi, Ei - Or};
+    }
+}
+
+// k_c2r_pre_dist: the same at G > 1 for rank g's block k = k0 + j, j < nl, with X_{H-k} from the
+// mirror exchange (Xm = rank G-1-g's block, X_{H-k} = Xm[nl - j] for j > 0, xx = X_{H-k0}, which
+// is X_H for rank 0); writes conj(Z_k) for the rank's own k only.
+template <typename R>
+__global__ void __launch_bounds__(256)
+k_c2r_pre_dist(const C2<R>* __restrict__ X, const C2<R>* __restrict__ Xm, const C2<R>* __restrict__ xx,
+               C2<R>* __restrict__ Zc, long long H, long long nl, long long k0) {
+    pdl_trigger();
+    pdl_wait();
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    for (long long j = (long long)blockIdx.x * blockDim.x + threadIdx.x; j < nl; j += stride) {
+        const long long k = k0 + j;
+        C2<R> a = X[j];
+        C2<R> xb = j == 0 ? xx[0] : Xm[nl - j];
+        if (k == 0) a.y = xb.y = R(0);     // X_0, X_H of a real signal are real: Im ignored (fmmfft.h)
+        const R Er = R(0.5) * (a.x + xb.x), Ei = R(0.5) * (a.y - xb.y);
+        const R Dr = R(0.5) * (a.x - xb.x), Di = R(0.5) * (a.y + xb.y);
+        R wr, wi;                                                        // w_N^{-k}
+        if constexpr (sizeof(R) == 4) {
+            float sn, cs;
+            sincospif((float)((double)k / (double)H), &sn, &cs);
+            wr = cs; wi = sn;
+        } else {
+            double sn, cs;
+            sincospi((double)k / (double)H, &sn, &cs);
+            wr = cs; wi = sn;
+        }
+        const R Or = wr * Dr - wi * Di, Oi = wr * Di + wi * Dr;
+        Zc[j] = C2<R>{Er - Oi, -(Ei + Or)};
     }
 }
 

@@ -104,7 +104,7 @@ class FmmFFT:
 
     # -- execution
     def __call__(self, x: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
-        half = self.N // 2 + 1
+        half = self.n_local // 2 + 1              # real plans: this rank's N/(2G) + 1 (virtual: N/2 + 1)
         n_in = half if self.real and self.inverse else self.n_local
         n_out = half if self.real and not self.inverse else self.n_local
         if x.dtype != self.in_dtype or not x.is_cuda or not x.is_contiguous() or x.numel() != n_in:

@@ -109,8 +109,9 @@ def test_flag_values_match_header(L):
                    "VIRTUAL_NCCL": L.FLAG_VIRTUAL_NCCL}
 
 
-def test_real_multi_gpu_unsupported(L):
-    # FMMFFT_FLAG_REAL is single-GPU: rejected before any device or communicator is touched
+def test_real_rejects_odd_length(L):
+    # FMMFFT_FLAG_REAL (any G, incl. G > 1 since round 2) needs an even real length: rejected before
+    # any device or communicator is touched
     h = ctypes.c_void_p()
-    st = L.lib.fmmfft_plan_ex(ctypes.byref(h), 1 << 21, 64, 2, 2, 16, 0, 64, 32 | 1)
-    assert st == L.UNSUPPORTED and b"G = 1" in L.lib.fmmfft_last_error() and not h.value
+    st = L.lib.fmmfft_plan_ex(ctypes.byref(h), (1 << 21) + 1, 64, 2, 2, 16, 0, 64, 32 | 1)
+    assert st == L.INVALID_VALUE and b"even" in L.lib.fmmfft_last_error() and not h.value

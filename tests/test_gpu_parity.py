@@ -333,6 +333,44 @@ def test_alternative_paths(F, monkeypatch, env, N, P, B, Q, G):
         assert rel(LL[:, :, 1:], st["L"][L]) < TOL_STAGE[prec]
 
 
+# ------------------------------------------------------------------ fast-convolution S2T (§8(f) NEXT-4)
+@pytest.mark.parametrize("N,P,B,Q,prec,G", [
+    (1 << 18, 64, 3, 16, "c64", 1),          # 64 boxes: 2 chunks of 32, periodic wrap at both ends
+    (1 << 18, 64, 3, 16, "c128", 1),
+    (1 << 20, 16, 4, 16, "c64", 1),          # 1024 boxes: several chunks per CTA
+    (1 << 20, 16, 4, 24, "c128", 1),
+    (1 << 20, 16, 3, 16, "c64", 2),          # virtual ranks: halo boxes at the rank edges
+    (1 << 20, 32, 3, 16, "c128", 4),
+])
+def test_s2t_fft(F, monkeypatch, N, P, B, Q, prec, G):
+    # T_near by per-box DFT_128, the three kernel spectra and the inverse DFT_128 equals the
+    # oracle's direct sum (Alg. 1 line 3) at the stage tolerance; p = 0 (C_0 = I) copies exactly
+    monkeypatch.setenv("FMMFFT_S2T", "fft")
+    plan, x, y = run(F, N, P, B, Q, prec, 64, G=G, virtual=G > 1, debug=G == 1)
+    assert plan.info["variant"] & 128                  # FMMFFT_VARIANT_S2T_FFT
+    assert rel(y, O.fft_radix2(x)) < TOL_E2E[prec]
+    if G == 1:
+        L = O.tree_levels(N, P, 64)
+        S = x.astype(np.complex128).reshape(2 ** L, 64, P)
+        Tn = t_near(plan, P, L, 64)
+        assert rel(Tn, O.stage_s2t(S, N, P)) < TOL_STAGE[prec]
+        assert np.array_equal(Tn[:, :, 0], x.reshape(2 ** L, 64, P)[:, :, 0])
+
+
+@pytest.mark.parametrize("kind", ["dmma", "simt"])
+def test_s2t_c128_direct_kernels(F, monkeypatch, kind):
+    # the complex128 direct-sum S2T kernels the fast convolution replaced as the default:
+    # k_s2t_dmma (FP64 tensor pipe) and k_near_up (DFMA), same stage parity
+    monkeypatch.setenv("FMMFFT_S2T", kind)
+    N, P, B, Q = 1 << 18, 64, 3, 16
+    plan, x, y = run(F, N, P, B, Q, "c128", 64, debug=True)
+    assert not plan.info["variant"] & 128
+    assert rel(y, O.fft_radix2(x)) < TOL_E2E["c128"]
+    L = O.tree_levels(N, P, 64)
+    S = x.astype(np.complex128).reshape(2 ** L, 64, P)
+    assert rel(t_near(plan, P, L, 64), O.stage_s2t(S, N, P)) < TOL_STAGE["c128"]
+
+
 # ------------------------------------------------------------------ large-M four-step FFT passes
 @pytest.mark.parametrize("N,P,prec,G,env", [
     (1 << 23, 2, "c64", 1, None),        # M = 2^22: column pass 2^11 + transposing row pass 2^11
@@ -468,9 +506,44 @@ def test_real_input_vs_oracle(F, N, P, B, Q, prec, direct):
 def test_real_rejects_unsupported(F):
     from paper_conf_sc_cecka17_b200._lib import FmmfftError
     with pytest.raises(FmmfftError):
-        F(N=1 << 13, P=16, G=2, virtual=True, real=True)
+        F(N=(1 << 13) + 1, P=16, real=True)                    # odd real length
     with pytest.raises(FmmfftError):
-        F(N=1 << 13, P=16, G=2, virtual=True, inverse=True, real=True)
+        F(N=3 << 12, P=16, G=2, virtual=True, real=True)       # N/2 not a power of two
+
+
+@pytest.mark.parametrize("N,P,G,prec,direct,transport", [
+    (1 << 17, 16, 2, "c64", False, "copy"),
+    (1 << 17, 32, 4, "c128", False, "copy"),
+    (1 << 18, 64, 8, "c64", False, "copy"),
+    (1 << 17, 16, 4, "c64", True, "copy"),      # the distributed six-step FFT (NEXT-3) underneath
+    (1 << 17, 16, 2, "c128", False, "nccl"),    # the mirror exchange through NCCL send / recv
+])
+def test_real_distributed(F, request, N, P, G, prec, direct, transport):
+    # real input at G > 1 (virtual ranks): the complex plan of N/2 block-distributed, then the
+    # mirror exchange (rank g <- rank G-1-g's block + one element) and the per-rank separation;
+    # the global output X_0..X_{N/2} (rank g's block at g N/(2G), X_{N/2} after the last block)
+    if transport == "nccl":
+        request.getfixturevalue("nccl_local")
+    rdt = np.float32 if prec == "c64" else np.float64
+    x = SI.real_uniform(0, N, dtype=rdt)
+    ref = O.rdft(x.astype(np.float64))
+    fwd = F(N=N, P=P, G=G, B=2, Q=16, precision=prec, direct=direct, real=True, virtual=True, transport=transport)
+    y = fwd(torch.from_numpy(x).cuda())
+    assert y.shape == (N // 2 + 1,)
+    assert rel(y.cpu().numpy(), ref) < TOL_E2E[prec]
+    assert blockwise_rel(y.cpu().numpy()[:-1], ref[:-1], G) < 2 * TOL_E2E[prec]
+    # complex-to-real inverse of the oracle's spectrum (non-real X_0 / X_{N/2} parts ignored)
+    X = ref.copy()
+    X[0] += 0.7j
+    X[-1] += 0.3j
+    inv = F(N=N, P=P, G=G, B=2, Q=16, precision=prec, direct=direct, real=True, inverse=True, virtual=True,
+            transport=transport)
+    z = inv(torch.from_numpy(X.astype(NPDT[prec])).cuda()).cpu().numpy()
+    assert z.shape == (N,)
+    assert np.linalg.norm(z - x) / np.linalg.norm(x) < TOL_E2E[prec]
+    # device round trip
+    w = inv(y).cpu().numpy()
+    assert np.linalg.norm(w - x) / np.linalg.norm(x) < 2 * TOL_E2E[prec]
 
 
 @pytest.mark.parametrize("N,P,B,Q,prec,direct", [

@@ -29,6 +29,41 @@ def test_virtual_ranks_match_global(N, P, B, Q, M_L, G):
     assert O.rel_l2(y, np.fft.fft(x)) < (3e-14 if Q >= 16 else 1e-9)   # M_L = 16: see test_oracle_fmm
 
 
+@pytest.mark.parametrize("N,P,B,Q,M_L,G", [
+    (1 << 13, 16, 2, 16, 16, 1),
+    (1 << 13, 16, 2, 16, 16, 2),
+    (1 << 15, 16, 2, 16, 16, 4),
+    (1 << 15, 16, 2, 12, 16, 8),
+])
+def test_real_input_virtual_ranks(N, P, B, Q, M_L, G):
+    # reading R18 at G ranks: the mirror exchange + per-rank even/odd separation equals the
+    # definition (eq. 1 for real x, first half: O.rdft, pinned to numpy.fft.rfft) and inverts
+    x = SI.real_uniform(0, N)
+    X = D.rdft_virtual(x, P, B, Q, M_L, G)
+    assert X.shape == (N // 2 + 1,)
+    ref = O.rdft(x)
+    assert O.rel_l2(X, ref) < (3e-14 if Q >= 16 else 1e-9)
+    assert abs(X[0].imag) < 1e-12 * abs(X[0]) + 1e-12 and abs(X[-1].imag) < 1e-12 * np.abs(X).max()
+    Xb = ref.copy()
+    Xb[0] += 0.7j                       # non-real DC / Nyquist parts are ignored by the inverse
+    Xb[-1] += 0.3j
+    xr = D.irdft_virtual(Xb, P, B, Q, M_L, G)
+    assert np.linalg.norm(xr - x) / np.linalg.norm(x) < (3e-14 if Q >= 16 else 1e-9)
+
+
+def test_mirror_exchange_pairs():
+    # every rank receives rank G-1-g's block and A[(G-g) H/G] (R2C: A[H] = A[0]; C2R: A[H] = X_H)
+    for G in (1, 2, 3, 4, 8):
+        nl = 5
+        A = np.arange(G * nl + 1) * (1 + 1j)                           # global A_0 .. A_H
+        for c2r in (False, True):
+            res = D._run_threads(G, lambda g, comm: D.mirror_exchange(A[g * nl:(g + 1) * nl], A[G * nl], g, G, comm, c2r))
+            for g, (mir, xtra) in enumerate(res):
+                assert np.array_equal(mir, A[(G - 1 - g) * nl:(G - g) * nl])
+                want = A[(G - g) * nl] if (c2r or g > 0) else A[0]
+                assert xtra == want, (G, c2r, g)
+
+
 def test_shards_are_slices_of_the_global_vector():
     N, G = 1 << 12, 4
     full = SI.complex_uniform(0, N)
@@ -82,8 +117,11 @@ def _gloo_worker(rank, world, port, q):
     try:
         N, P, B, Q, M_L = 1 << 14, 16, 3, 16, 16
         x = SI.shard(N, world, rank)
-        y = D.fmmfft_rank(x, N, P, B, Q, M_L, rank, world, GlooGroup(torch, dist))
-        q.put((rank, y))
+        comm = GlooGroup(torch, dist)
+        y = D.fmmfft_rank(x, N, P, B, Q, M_L, rank, world, comm)
+        xr = SI.real_uniform(0, 2 * N)[rank * N:(rank + 1) * N]       # 2N reals: H = N
+        X = D.rdft_rank(xr, 2 * N, P, B, Q, M_L, rank, world, comm)
+        q.put((rank, (y, X)))
     finally:
         dist.destroy_process_group()
 
@@ -109,7 +147,10 @@ def test_gloo_two_processes():
         p.join(timeout=60)
         assert p.exitcode == 0
     N = 1 << 14
-    y = np.concatenate([got[0], got[1]])
+    y = np.concatenate([got[0][0], got[1][0]])
     x = SI.complex_uniform(0, N)
     assert O.rel_l2(y, O.fmmfft(x, 16, 3, 16, 16)) < 1e-14
     assert O.rel_l2(y, O.fft_radix2(x)) < 3e-14
+    # real input over the two processes: the mirror exchange through gloo (R18)
+    X = np.concatenate([got[0][1], got[1][1]])
+    assert O.rel_l2(X, O.rdft(SI.real_uniform(0, 2 * N))) < 3e-14
