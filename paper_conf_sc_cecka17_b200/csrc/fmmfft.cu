@@ -200,6 +200,7 @@ struct RankBufs {
     void* haloR = nullptr;   // S box nb  (G > 1)
     void* r = nullptr;       // [P] reductions
     void* dc = nullptr;      // [P/G] the k1 = 0 outputs of this rank's M-FFT rows (k_dc_bins, R19)
+    void* r0p = nullptr;     // [(P-1) top_cl] double2 partial sums of r_0 (wide trees with the cluster top)
     void* cin = nullptr;     // conj(in) (inverse plans)
     void* rz = nullptr;      // Z = F_{N/2} z (real-input plans, FMMFFT_FLAG_REAL)
     void* mir = nullptr;     // real plans, G > 1: the mirror block (rank G-1-g's Z or X block)
@@ -239,6 +240,8 @@ struct fmmfft_plan_s {
     std::vector<void*> m2l_pmaj;     // p-major copies for the fused per-p tree (G = 1), by level
     bool tree_p = false;             // use k_tree_p for the far field
     int tree_cl = 1;                 // k_tree_pc: CTAs per FMM (cluster), 1 = not used
+    int top_L = 0;                   // > 0: wide tree (G = 1) whose levels B..top_L run on k_tree_pc
+    int top_cl = 0;                  //   with clusters of top_cl CTAs; levels > top_L per level
     int fs_lc1 = 0, fs_lc2 = 0, fs_lr = 0;   // four-step large-M FFT: column pass bits (2nd: 0 = none), row pass bits
     bool inverse = false;            // FMMFFT_FLAG_INVERSE: x = F_N^{-1} y
     bool real = false;               // FMMFFT_FLAG_REAL: N (below) is the complex length H = N_real / 2
@@ -525,6 +528,7 @@ static fmmfft_status_t alloc_rank(fmmfft_plan_s* p, RankBufs& rb) {
     }
     if ((st = dalloc(p, &rb.r, (size_t)p->P * e))) return st;
     if ((st = dalloc(p, &rb.dc, (size_t)(p->P / p->G) * e))) return st;
+    if (p->top_L && (st = dalloc(p, &rb.r0p, (size_t)(p->P - 1) * p->top_cl * 16))) return st;
     rb.Mpad.assign(p->L + 1, nullptr);
     rb.Lloc.assign(p->L + 1, nullptr);
     rb.Mfull.assign(p->L + 1, nullptr);
@@ -618,9 +622,14 @@ static fmmfft_status_t init_kernel_attrs() {
         if constexpr (sizeof(R) == 4) {
             set((const void*)k_tree_pc<16, 512, 2>);
             set((const void*)k_tree_pc<8, 512, 2>);
+            set((const void*)k_tree_pc<16, 512, 4>);
+            set((const void*)k_tree_pc<8, 512, 4>);
+            set((const void*)k_tree_pc<16, 512, 8>);
+            set((const void*)k_tree_pc<8, 512, 8>);
         }
         if constexpr (sizeof(R) == 4) { set((const void*)k_s2t_tc<1>); set((const void*)k_s2t_tc<2>); }
         set((const void*)k_s2t_fft<R>);
+        set((const void*)k_s2m_w<R>);
         set((const void*)k_base_sg<R, 4, sizeof(R) == 4 ? 8 : 4, 4>);
         for (int lp = 1; lp <= 5; ++lp)
             dispatch<1, 2, 3, 4, 5>(lp, [&](auto v) {
@@ -684,13 +693,14 @@ static size_t tree_p_smem(const fmmfft_plan_s* p, int threads) {
 }
 
 // shared memory of k_tree_pc (cluster of CL CTAs per FMM)
-static size_t tree_pc_smem(const fmmfft_plan_s* p, int CL) {
+static size_t tree_pc_smem(const fmmfft_plan_s* p, int CL, int Lt = -1) {
+    const int L = Lt >= 0 ? Lt : p->L;                  // the tree's (top) leaf level
     const size_t Q = p->Q, QQ = Q * Q, nbB = (size_t)1 << p->B;
     const size_t tabB = (nbB - 3) * QQ;
     auto H = [&](int l) { return ((size_t)1 << l) / CL; };
-    size_t cplx = 32 + nbB * Q + (nbB / CL) * Q + H(p->L) * Q + (p->L > 0 ? H(p->L - 1) : 0) * Q;
-    for (int l = p->B + 1; l <= p->L; ++l) cplx += (H(l) + 6) * Q;
-    return (2 * QQ + tabB + (size_t)(p->L - p->B) * 4 * QQ) * 4 + QQ * 8 + cplx * 8;
+    size_t cplx = 32 + nbB * Q + (nbB / CL) * Q + H(L) * Q + (L > 0 ? H(L - 1) : 0) * Q;
+    for (int l = p->B + 1; l <= L; ++l) cplx += (H(l) + 6) * Q;
+    return (2 * QQ + tabB + (size_t)(L - p->B) * 4 * QQ) * 4 + QQ * 8 + cplx * 8;
 }
 
 // ------------------------------------------------------------------ execute
@@ -889,6 +899,20 @@ struct Exec {
     fmmfft_status_t near_up() {
         fmmfft_status_t st;
         const int PCs = std::min(p->P, sizeof(R) == 4 ? 32 : 16);
+        constexpr int PCW = s2mw_pc<R>();
+        // complex64 (complex128's S2M is DFMA-bound with Q = 24: k_s2m measured faster, 1.68 vs 2.12 ms)
+        if (sizeof(R) == 4 && p->M_L == 64 && p->P % PCW == 0 && !getenv("FMMFFT_S2M_OLD")) {   // warp-per-box S2M (k_s2m_w)
+            const int Qp = (p->Q + 3) / 4 * 4;
+            const long long tasks = (long long)p->nb * (p->P / PCW);
+            const int bpw = (int)std::max<long long>(1, std::min<long long>(8, tasks / (S2MW_WARPS * 148 * 4)));
+            const dim3 grid((unsigned)((p->nb + (long long)S2MW_WARPS * bpw - 1) / ((long long)S2MW_WARPS * bpw)), (unsigned)(p->P / PCW));
+            for (RankBufs& rb : p->ranks) {
+                const C* S = in[p->virt ? rb.g : 0];
+                launch_pdl(k_s2m_w<R>, grid, S2MW_WARPS * 32, s2mw_smem<R>(Qp), s, S, interior(rb.Mpad[p->L]), (const R*)p->s2mT,
+                           p->P, p->Q, (C*)rb.Sp, (C*)rb.Tn, p->nb, (int)p->pmaj, bpw);
+                LAUNCH_CHECK();
+            }
+        } else
         for (RankBufs& rb : p->ranks) {
             const C* S = in[p->virt ? rb.g : 0];
             const int Qp = (p->Q + 3) / 4 * 4;
@@ -931,21 +955,21 @@ struct Exec {
         }
         if constexpr (sizeof(R) == 4) {
             if (p->s2t_tc) {                                   // tensor cores (tcgen05, 3xTF32)
-                const int ntile = p->nb / S2TC_BOXES;
-                // tiles per CTA: the fewest that keep the grid within one wave of 148 SMs
-                // (one CTA per SM: TMEM + ~180 KB of shared memory)
-                const int cpp = std::max(1, 148 / (p->P - 1));             // CTAs per p
-                int tpc = (ntile + cpp - 1) / cpp;
+                const long long work = (long long)(p->P - 1) * (p->nb / S2TC_BOXES);
+                // one CTA per SM (TMEM + ~180 KB of shared memory); the (p, tile) items split evenly
+                // over (P - 1) floor(148 / (P - 1)) CTAs, so a CTA's run stays within one p (B_p
+                // loaded once) and the few SMs left over run the far field meanwhile (measured:
+                // all 148 SMs on S2T, with B_p reloads, was 334 -> 354 us at cfg3)
+                const int ctas = (int)std::min<long long>((long long)(p->P - 1) * std::max(1, 148 / (p->P - 1)), work);
                 for (RankBufs& rb : p->ranks) {
-                    const dim3 grid((unsigned)((ntile + tpc - 1) / tpc), (unsigned)(p->P - 1));
                     // several tiles per CTA: A chunks prefetched two ahead; one tile: one ahead (the
                     // first chunk's loads alone, so the first MMAs start sooner)
-                    if (tpc > 1)
-                        launch_pdl(k_s2t_tc<2>, grid, S2TC_THREADS, s2tc_smem_bytes(), side(), (const C*)rb.Sp, (const C*)rb.haloL,
-                                   (const C*)rb.haloR, (float*)rb.Tn, (const float*)p->toep, p->P, p->nb, p->G, tpc);
+                    if (work > ctas)
+                        launch_pdl(k_s2t_tc<2>, dim3((unsigned)ctas), S2TC_THREADS, s2tc_smem_bytes(), side(), (const C*)rb.Sp,
+                                   (const C*)rb.haloL, (const C*)rb.haloR, (float*)rb.Tn, (const float*)p->toep, p->P, p->nb, p->G);
                     else
-                        launch_pdl(k_s2t_tc<1>, grid, S2TC_THREADS, s2tc_smem_bytes(), side(), (const C*)rb.Sp, (const C*)rb.haloL,
-                                   (const C*)rb.haloR, (float*)rb.Tn, (const float*)p->toep, p->P, p->nb, p->G, tpc);
+                        launch_pdl(k_s2t_tc<1>, dim3((unsigned)ctas), S2TC_THREADS, s2tc_smem_bytes(), side(), (const C*)rb.Sp,
+                                   (const C*)rb.haloL, (const C*)rb.haloR, (float*)rb.Tn, (const float*)p->toep, p->P, p->nb, p->G);
                     LAUNCH_CHECK();
                 }
                 if ((st = mark_on(p->ev_s2t[1], side()))) return st;
@@ -1099,6 +1123,7 @@ struct Exec {
             a.B = p->B;
             a.dbg = (p->flags & FMMFFT_FLAG_DEBUG) ? 1 : 0;
             a.pmaj = p->pmaj ? 1 : 0;
+            a.p0 = 1;
             const int tabB = ((1 << p->B) - 3) * p->Q * p->Q;
             // complex64, Q = 16 or 8: each FMM on a cluster of 2 CTAs (k_tree_pc)
             if constexpr (sizeof(R) == 4) {
@@ -1123,13 +1148,44 @@ struct Exec {
         return FMMFFT_SUCCESS;
     }
 
+    // ---- wide trees (G = 1): levels B..top_L of each FMM on a cluster (k_tree_pc with top_L as
+    // its leaf level: M^{top_L} from the per-level M2M in, L^{top_L} for the per-level M2L out)
+    fmmfft_status_t tree_top() {
+        for (RankBufs& rb : p->ranks) {
+            TreePArgs a{};
+            for (int lev = p->B; lev <= p->top_L; ++lev) {
+                a.M[lev] = interior(rb.Mpad[lev]);
+                a.Lx[lev] = rb.Lloc[lev];
+                a.tab[lev] = p->m2l_pmaj[lev];
+            }
+            a.r = rb.r;
+            a.L = p->top_L;
+            a.B = p->B;
+            a.dbg = (p->flags & FMMFFT_FLAG_DEBUG) ? 1 : 0;
+            a.pmaj = 0;
+            a.p0 = 1;
+            a.r0part = rb.r0p;                              // r_0 (R19): partial sums of M^{top_L} slot 0
+            const int tabB = ((1 << p->B) - 3) * p->Q * p->Q;
+            const size_t smem = tree_pc_smem(p, p->top_cl, p->top_L);
+            const unsigned grid = (unsigned)((p->P - 1) * p->top_cl);
+            auto go = [&](auto cl) {
+                constexpr int CL = decltype(cl)::value;
+                if (p->Q == 16) launch_cluster(k_tree_pc<16, 512, CL>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
+                else            launch_cluster(k_tree_pc<8, 512, CL>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
+            };
+            dispatch<2, 4, 8>(p->top_cl, go);
+            LAUNCH_CHECK();
+        }
+        return FMMFFT_SUCCESS;
+    }
+
     // ---- m2m on own boxes, l = L-1 .. l_g
     fmmfft_status_t m2m_local() {
         if (p->tree_p) return FMMFFT_SUCCESS;
         fmmfft_status_t st;
         for (RankBufs& rb : p->ranks) {
             auto outs = [&](int l) -> void* { return interior(rb.Mpad[l]); };
-            if ((st = launch_up(interior(rb.Mpad[p->L]), p->L, p->lg, nb_at(p->L), outs))) return st;
+            if ((st = launch_up(interior(rb.Mpad[p->L]), p->L, p->top_L ? p->top_L : p->lg, nb_at(p->L), outs))) return st;
         }
         return FMMFFT_SUCCESS;
     }
@@ -1189,6 +1245,8 @@ struct Exec {
     // ---- top: replicated levels l_g .. B
     fmmfft_status_t top() {
         if (p->tree_p) return tree_p();
+        if constexpr (sizeof(R) == 4)
+            if (p->top_L) return tree_top();
         fmmfft_status_t st;
         for (RankBufs& rb : p->ranks) {
             const int g = grank(rb);
@@ -1250,6 +1308,7 @@ struct Exec {
 
     fmmfft_status_t down() {
         if (p->L == p->B || p->tree_p) return FMMFFT_SUCCESS;
+        if (p->top_L) return p->top_L < p->L ? down_levels(p->top_L + 1) : FMMFFT_SUCCESS;
         int lnew = lvl_first();
         if (narrow_ok()) {                           // k_down_narrow up to the widest level that fits
             int lnar = p->B, nmax = 0;
@@ -1542,7 +1601,8 @@ struct Exec {
                 m0_stride = p->pmaj ? 1 : p->P;
             }
             launch_pdl(k_dc_bins<R>, (unsigned)((rows + 7) / 8), 256, 0, side(), (C*)rb.dc, (const C*)rb.r, m0, m0_n,
-                       m0_stride, p->P, rows, grank(rb) * rows, (long long)p->M);
+                       m0_stride, p->P, rows, grank(rb) * rows, (long long)p->M, (const double2*)rb.r0p,
+                       p->top_L ? (p->P - 1) * p->top_cl : 0);
             LAUNCH_CHECK();
         }
         CUDA_TRY(cudaEventRecord(p->dc_join, side()));
@@ -2001,6 +2061,23 @@ static fmmfft_status_t plan_complex(fmmfft_plan_t* plan, long long N, int P, int
         // complex64, Q = 8 / 16: each FMM's tree on a cluster of 2 CTAs (k_tree_pc); else one CTA
         // per FMM (k_tree_p)
         if (p->tree_p && precision == FMMFFT_C64 && (Q == 16 || Q == 8) && tree_pc_smem(p, 2) <= (size_t)optin) p->tree_cl = 2;
+        // wide trees at G = 1 (complex64, Q = 8 / 16): the levels below the first wide level (the
+        // per-level kernels' launch-latency-bound top: k_up, k_base, k_tree_down) as ONE k_tree_pc
+        // launch, each FMM's top subtree on a cluster of 8 (else 4, 2) CTAs, levels B..top_L
+        // entirely on chip; FMMFFT_TOP=w keeps the per-level kernels
+        const char* et = getenv("FMMFFT_TOP");
+        if (!p->tree_p && G == 1 && precision == FMMFFT_C64 && (Q == 16 || Q == 8) && L > B && !(et && et[0] == 'w') &&
+            (P % 8) == 0) {
+            int lt = L;                                     // = lvl_first - 1 (Exec::lvl_first at G = 1)
+            for (int lev = B + 1; lev <= L; ++lev)
+                if ((1LL << lev) >= 64 && (long long)((1LL << lev) / 32) * (P / 8) >= 148) { lt = lev - 1; break; }
+            for (int cl : {8, 4, 2})
+                if (lt > B && (2LL << B) >= 2LL * cl && tree_pc_smem(p, cl, lt) <= (size_t)optin) {
+                    p->top_L = lt;
+                    p->top_cl = cl;
+                    break;
+                }
+        }
     }
     // S2T kernel: complex64 with M_L = 64 and whole 128-box tiles per rank -> tensor cores
     // (k_s2t_tc, 3xTF32 on tcgen05); other M_L = 64 plans (32-box chunks) -> the fast convolution

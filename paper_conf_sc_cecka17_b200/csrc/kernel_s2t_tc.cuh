@@ -16,7 +16,10 @@
 // Precision: 3xTF32, T = Ahi Bhi + Ahi Blo + Alo Bhi accumulated in fp32 in tensor memory (plain
 // TF32 misses the 1e-5 bound): 9 MMAs (M=128, N=64, K=8) per K step and component.
 //
-// CTA = (FMM p, run of 128-box tiles), warp-specialised, 9 warps:
+// CTA = a contiguous run of (FMM p, 128-box tile) work items — (p - 1) ntile + t, split evenly
+// over one CTA per SM, so every SM gets the same number of tiles (a run crosses at most a few p;
+// the operator B_p is reloaded when p changes, after the previous tile's MMAs completed) —
+// warp-specialised, 9 warps:
 //   warps 0-3  build A (re/im x hi/lo, K chunks of 16 in a 2-slot ring) from the p-major copy
 //              S'[p][b][m] (the next chunk prefetched into registers); halo rows from the
 //              neighbouring boxes (periodic wrap at G = 1, the halo buffers at rank edges);
@@ -69,7 +72,7 @@ __host__ __device__ constexpr size_t s2tc_smem_bytes() { return (size_t)S2tcSmem
 template <int PF>                                          // A-chunk prefetch distance (1 or 2)
 __global__ void __launch_bounds__(S2TC_THREADS, 1)
 k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const float2* __restrict__ haloR,
-         float* __restrict__ Tn, const float* __restrict__ toep, int P, int nb, int G, int tiles_per_cta) {
+         float* __restrict__ Tn, const float* __restrict__ toep, int P, int nb, int G) {
     pdl_trigger();
     pdl_wait();
     STAMP(0);
@@ -86,14 +89,12 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
     uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(smem_tc + S2tcSmem::TSLOT);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int p = blockIdx.y + 1;
     const int ntile = nb / S2TC_BOXES;
-    const int t0 = blockIdx.x * tiles_per_cta;
-    const int t1 = min(ntile, t0 + tiles_per_cta);
-    if (t0 >= t1) return;
-    const int nit = t1 - t0;
+    const long long W = (long long)(P - 1) * ntile;              // work items (p - 1) ntile + t
+    const int w0 = (int)(W * blockIdx.x / gridDim.x), w1 = (int)(W * (blockIdx.x + 1) / gridDim.x);
+    if (w0 >= w1) return;
+    const int nit = w1 - w0;
     const size_t pblk = (size_t)nb * 64;                         // elements per p block of S' / T
-    const float2* spp = Sp + (size_t)p * pblk;
 
     if (tid == 0) {
         for (int k = 0; k < 12; ++k) tc::mbar_init(&bar[k], (k == 4 || k == 5 || k >= 10) ? 128u : 1u);
@@ -111,7 +112,8 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
         // item j: row r = idx >> 2 (box b0 - 1 + r), k4 = idx & 3, idx = tid + 128 j < 4 x 130
         constexpr int NJ = (4 * S2TC_ROWS + 127) / 128;          // 5
         float4 sv[2][NJ][2];                                     // two chunks in flight (prefetch distance 2)
-        auto load_chunk = [&](float4 (&svb)[NJ][2], int t, int kc) {
+        auto load_chunk = [&](float4 (&svb)[NJ][2], int p, int t, int kc) {
+            const float2* spp = Sp + (size_t)p * pblk;
 #pragma unroll
             for (int j = 0; j < NJ; ++j) {
                 const int idx = tid + 128 * j;
@@ -136,9 +138,12 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
                 }
             }
         };
-        load_chunk(sv[0], t0, 0);
-        if (PF == 2) load_chunk(sv[1], t0, 1);
+        // (p, t) of the tile being built and of the next one (no division in the pacing loop)
+        int pc = w0 / ntile + 1, tc_ = w0 - (pc - 1) * ntile;
+        load_chunk(sv[0], pc, tc_, 0);
+        if (PF == 2) load_chunk(sv[1], pc, tc_, 1);
         for (int it = 0; it < nit; ++it) {
+            const int pn = tc_ + 1 == ntile ? pc + 1 : pc, tn = tc_ + 1 == ntile ? 0 : tc_ + 1;
 #pragma unroll
             for (int kc = 0; kc < S2TC_NKC; ++kc) {
                 const int gi = it * S2TC_NKC + kc, slot = gi & 1, use = gi >> 1;
@@ -170,25 +175,41 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
                 tc::mbar_arrive(&cfull[slot]);
                 if (it < 2) STAMP(41 + 4 * it + kc);
                 // prefetch chunk kc + PF (into the buffer just consumed when PF = 2; S2TC_NKC is even)
-                if (kc + PF < S2TC_NKC) load_chunk(sv[(kc + PF) & 1], t0 + it, kc + PF);
-                else if (it + 1 < nit) load_chunk(sv[(kc + PF) & 1], t0 + it + 1, kc + PF - S2TC_NKC);
+                if (kc + PF < S2TC_NKC) load_chunk(sv[(kc + PF) & 1], pc, tc_, kc + PF);
+                else if (it + 1 < nit) load_chunk(sv[(kc + PF) & 1], pn, tn, kc + PF - S2TC_NKC);
             }
+            pc = pn;
+            tc_ = tn;
         }
     } else if (warp == 8) {
         // ------------------------------------------------------------ operator loads + MMA issue
         if (lane == 0) {
-            const float* tp = toep + (size_t)p * S2TC_TAB_FLOATS_PER_P;
-            for (int kc = 0; kc < S2TC_NKC; ++kc) {              // B chunk kc: k4 in [4 kc, 4 kc + 4), hi and lo
-                tc::mbar_expect_tx(&bfull[kc], 4 * S2TC_B_K4N);
-                tc::bulk_g2s(Bsm + kc * 4 * S2TC_B_K4N, tp + kc * S2TC_B_K4N, 4 * S2TC_B_K4N, &bfull[kc]);
-            }
+            auto load_B = [&](int p) {
+                const float* tp = toep + (size_t)p * S2TC_TAB_FLOATS_PER_P;
+                for (int kc = 0; kc < S2TC_NKC; ++kc) {          // B chunk kc: k4 in [4 kc, 4 kc + 4), hi and lo
+                    tc::mbar_expect_tx(&bfull[kc], 4 * S2TC_B_K4N);
+                    tc::bulk_g2s(Bsm + kc * 4 * S2TC_B_K4N, tp + kc * S2TC_B_K4N, 4 * S2TC_B_K4N, &bfull[kc]);
+                }
+            };
+            int pcur = w0 / ntile + 1, bphase = 0;
+            bool bnew = true;                                    // wait for the B chunks at the next tile
+            load_B(pcur);
             constexpr uint32_t IDESC128 = tc::idesc_tf32(128, 128), IDESC64 = tc::idesc_tf32(128, 64);
             for (int it = 0; it < nit; ++it) {
                 const int buf = it & 1;
+                const int pit = (w0 + it) / ntile + 1;
+                if (pit != pcur) {                               // next FMM: reload B_p once tile it-1's MMAs completed
+                    tc::mbar_wait(&afull[(it - 1) & 1], ((it - 1) >> 1) & 1);
+                    tc::tc_fence_after();
+                    pcur = pit;
+                    bphase ^= 1;
+                    bnew = true;
+                    load_B(pcur);
+                }
                 if (it >= 2) tc::mbar_wait(&aempty[buf], ((it >> 1) + 1) & 1);   // epilogue of tile it-2 done
                 for (int kc = 0; kc < S2TC_NKC; ++kc) {
                     const int gi = it * S2TC_NKC + kc, slot = gi & 1, use = gi >> 1;
-                    if (it == 0) tc::mbar_wait(&bfull[kc], 0);
+                    if (bnew) tc::mbar_wait(&bfull[kc], bphase);
                     tc::mbar_wait(&cfull[slot], use & 1);
                     tc::tc_fence_after();
                     const unsigned char* As = Asm + slot * S2TC_A_SLOT;
@@ -213,6 +234,7 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
                     tc::mma_commit(&cempty[slot]);
                     if (it < 2) STAMP(2 + 4 * it + kc);
                 }
+                bnew = false;
                 tc::mma_commit(&afull[buf]);
             }
         }
@@ -222,7 +244,8 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
         const int q = warp & 3;
         float* xt = Xt + q * 32 * 33;
         for (int it = 0; it < nit; ++it) {
-            const int t = t0 + it, buf = it & 1;
+            const int w = w0 + it, buf = it & 1;
+            const int p = w / ntile + 1, t = w - (p - 1) * ntile;
             if (it < 4) STAMP(20 + 4 * it);
             tc::mbar_wait(&afull[buf], (it >> 1) & 1);
             tc::tc_fence_after();

@@ -708,7 +708,7 @@ k_conj_scale(const C2<R>* in, C2<R>* out, long long n, R scale) {   // in == out
 template <typename R>
 __global__ void __launch_bounds__(256)
 k_dc_bins(C2<R>* __restrict__ y, const C2<R>* __restrict__ r, const C2<R>* __restrict__ m0, long long m0_n,
-          long long m0_stride, int P, int rows, int row0, long long M) {
+          long long m0_stride, int P, int rows, int row0, long long M, const double2* __restrict__ r0part, int nr0part) {
     pdl_trigger();
     __shared__ double2 red[8];
     __shared__ double2 rr[1024];                                  // r_p (r_0 replaced), then summed
@@ -717,6 +717,14 @@ k_dc_bins(C2<R>* __restrict__ y, const C2<R>* __restrict__ r, const C2<R>* __res
     for (int j = tid; j < P; j += blockDim.x) tw[j] = twiddle_d(j, P);
     pdl_wait();
     for (int j = tid; j < P; j += blockDim.x) rr[j] = make_double2((double)r[j].x, (double)r[j].y);
+    if (nr0part > 0) {                                            // r_0 from the tree kernel's partial sums
+        __syncthreads();
+        if (tid == 0) {
+            double2 t = make_double2(0.0, 0.0);
+            for (int k = 0; k < nr0part; ++k) { t.x += r0part[k].x; t.y += r0part[k].y; }   // fixed order
+            rr[0] = t;
+        }
+    }
     if (m0 != nullptr) {                                          // r_0 = sum of M^L slot 0
         double2 a = make_double2(0.0, 0.0);
         for (long long i0 = tid; i0 < m0_n; i0 += 8LL * blockDim.x) {   // 8 independent loads in flight

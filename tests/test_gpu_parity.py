@@ -87,7 +87,8 @@ def test_cfg1_c128_matches_oracle_and_direct_dft(F):
 
 # ------------------------------------------------------------------ stage by stage
 @pytest.mark.parametrize("prec", ["c64", "c128"])
-@pytest.mark.parametrize("N,P,B,Q,M_L", [(1 << 16, 16, 2, 16, 32), (1 << 18, 64, 3, 16, 64)])
+@pytest.mark.parametrize("N,P,B,Q,M_L", [(1 << 16, 16, 2, 16, 32), (1 << 18, 64, 3, 16, 64),
+                                         (1 << 20, 16, 4, 16, 16)])   # L = 12: per-level 12, cluster top 4..11 (c64)
 def test_stages_match_oracle(F, prec, N, P, B, Q, M_L):
     plan, x, y = run(F, N, P, B, Q, prec, M_L, debug=True)
     L = O.tree_levels(N, P, M_L)
@@ -307,7 +308,8 @@ def test_real_full_size_sampled(F):
 # ------------------------------------------------------------------ alternative kernel paths
 @pytest.mark.parametrize("env", [
     {"FMMFFT_S2T": "simt"},      # S2T on the FFMA2 SIMT kernel (k_near_up) instead of tcgen05
-    {"FMMFFT_TREE": "w"},        # far field as wide per-level kernels (k_up, k_base, k_tree_down + k_m2l_lvl)
+    {"FMMFFT_TREE": "w", "FMMFFT_TOP": "w"},   # far field as wide per-level kernels (k_up, k_base, k_tree_down + k_m2l_lvl)
+    {"FMMFFT_TREE": "w"},        # per-level kernels below, the top subtree of each FMM on a k_tree_pc cluster
     {"FMMFFT_NO_GRAPH": "1"},    # eager launches instead of a CUDA graph
     {"FMMFFT_MFFT": "pass"},     # multi-pass M-point FFT (k_fft_pass) instead of k_fft_row
     {"FMMFFT_MFFT": "fs"},       # four-step M-point FFT (k_fft_col + k_fft_rowt) instead of k_fft_row
