@@ -129,7 +129,8 @@ def load_traffic(workload: str, G: int, kernel: str):
         return None
 
 
-def stage_rooflines(N, P, B, Q, M_L, G, L, prec, tree_fused, s2t_tc, mfft_kernel):
+def stage_rooflines(N, P, B, Q, M_L, G, L, prec, tree_fused, s2t_tc, mfft_kernel, top_L=0, s2t_fft=False,
+                    s2m_w=False):
     """Algorithmic work per execute of each stage, per rank, restated from PAPER.md §5.1
     (P:1159-1174): W = flops (a complex-data x real-operator multiply-add is 2C = 4 real flops),
     D = algorithmic HBM bytes (each operand read once, each result written once). Returns
@@ -145,14 +146,27 @@ def stage_rooflines(N, P, B, Q, M_L, G, L, prec, tree_fused, s2t_tc, mfft_kernel
     down = 2 * C * fmm * Q * Q * 4 * dn
     base = 2 * C * fmm * Q * Q * 2 ** B * (2 ** B - 3) / G
     exp_b = Q * fmm * esz                                          # one box's expansions, all FMMs
+    # S2T as the fast convolution (k_s2t_fft): per (box, p) a forward and an inverse 128-point FFT
+    # (5 n log2 n each) and 3 complex products per frequency — the flops that kernel performs
+    s2t = (("k_s2t_fft", (2 * 5 * 128 * 7 + 3 * 128 * 8) * nb * fmm, 2 * nl * esz) if s2t_fft else
+           ("k_s2t_tc" if s2t_tc else "k_near_up", 6 * C * M_L * M_L * nb * fmm, 2 * nl * esz))
     out = {
-        "s2m": ("k_s2m", 2 * C * M_L * nb * fmm * Q, nl * esz + nb * exp_b),
-        "s2t": ("k_s2t_tc" if s2t_tc else "k_near_up", 6 * C * M_L * M_L * nb * fmm, 2 * nl * esz),
+        "s2m": ("k_s2m_w" if s2m_w else "k_s2m", 2 * C * M_L * nb * fmm * Q, nl * esz + nb * exp_b),
+        "s2t": s2t,
         "post_pfft": ("k_post_pfft", 2 * C * M_L * Q * nb * fmm + 5 * nl * math.log2(P), 2 * nl * esz + nb * exp_b),
         "mfft": (mfft_kernel, 5 * nl * math.log2(N // P), 2 * nl * esz),
     }
     if tree_fused:
         out["top"] = ("k_tree_pc", m2m + down + base, 2 * nb * exp_b)
+    elif top_L:
+        # wide levels per level; levels B..top_L of each FMM in one cluster kernel (k_tree_pc)
+        up_w = sum(2 ** l for l in range(top_L, L)) / G
+        dn_w = sum(2 ** l for l in range(top_L + 1, L + 1)) / G
+        m2m_w = 2 * C * fmm * Q * Q * 2 * up_w
+        down_w = 2 * C * fmm * Q * Q * 4 * dn_w
+        out["m2m"] = ("k_m2m_lvl", m2m_w, 3 * up_w * exp_b)
+        out["top"] = ("k_tree_pc", (m2m - m2m_w) + (down - down_w) + base, 2 * 2 ** top_L / G * exp_b)
+        out["down"] = ("k_m2l_lvl", down_w, 3 * dn_w * exp_b)
     else:
         out["m2m"] = ("k_m2m_lvl + k_up", m2m, 3 * up * exp_b)
         out["top"] = ("k_base", base, 2 * 2 ** B * exp_b)
@@ -277,7 +291,9 @@ def roofline_table(stages, N, P, B, Q, M_L, G, info, prec, workload, virt):
     mk = "k_fft_row" if v & 4 else "k_fft_col + k_fft_rowt" if v & 8 else "k_fft_pass"
     s2t_tc = bool(v & 2)
     rl = {}
-    for name, (kname, W, D) in stage_rooflines(N, P, B, Q, M_L, G, info["L"], prec, bool(v & 1), s2t_tc, mk).items():
+    for name, (kname, W, D) in stage_rooflines(N, P, B, Q, M_L, G, info["L"], prec, bool(v & 1), s2t_tc, mk,
+                                               info.get("top_level", 0) if v & 512 else 0, bool(v & 128),
+                                               bool(v & 256)).items():
         t = stages.get(name)
         if not t or t != t:
             continue

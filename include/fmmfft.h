@@ -189,10 +189,15 @@ typedef struct {
     size_t workspace_bytes; /* device bytes owned by the plan (all virtual ranks)   */
     int kernels_per_execute;/* kernels this library launched in the last execute (0 before) */
     unsigned variant;       /* kernel variants the plan chose: FMMFFT_VARIANT_* bits below  */
+    int top_level;          /* FMMFFT_VARIANT_TOP_CLUSTER: levels B..top_level of every FMM run
+                               in one cluster kernel, levels above it per level (else 0)  */
 } fmmfft_info_t;
 
 #define FMMFFT_VARIANT_TREE_FUSED 1u  /* far field as one per-FMM kernel (G = 1, tree fits smem) */
 #define FMMFFT_VARIANT_S2T_TC     2u  /* near field on tcgen05 tensor cores (3xTF32)             */
+#define FMMFFT_VARIANT_S2M_WARP 256u  /* S2M (+ the S' copy) one warp per box (k_s2m_w)            */
+#define FMMFFT_VARIANT_TOP_CLUSTER 512u /* wide tree (G = 1): the top levels of each FMM on a CTA
+                                         cluster (k_tree_pc), the wide levels per level            */
 #define FMMFFT_VARIANT_S2T_FFT  128u  /* near field as a fast convolution: per-box DFT_128, 3
                                          kernel spectra, inverse DFT_128 (k_s2t_fft, NEXT-4)       */
 #define FMMFFT_VARIANT_ROW_FFT1   4u  /* M-point FFTs as one single-pass kernel per row        */

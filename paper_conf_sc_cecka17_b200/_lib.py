@@ -28,7 +28,7 @@ class Info(ctypes.Structure):
                 ("Q", ctypes.c_int), ("M_L", ctypes.c_int), ("L", ctypes.c_int), ("precision", ctypes.c_int),
                 ("M", ctypes.c_longlong), ("level_gather", ctypes.c_int), ("n_stages", ctypes.c_int),
                 ("workspace_bytes", ctypes.c_size_t), ("kernels_per_execute", ctypes.c_int),
-                ("variant", ctypes.c_uint)]
+                ("variant", ctypes.c_uint), ("top_level", ctypes.c_int)]
 
 
 class Tune(ctypes.Structure):

@@ -242,6 +242,7 @@ struct fmmfft_plan_s {
     int tree_cl = 1;                 // k_tree_pc: CTAs per FMM (cluster), 1 = not used
     int top_L = 0;                   // > 0: wide tree (G = 1) whose levels B..top_L run on k_tree_pc
     int top_cl = 0;                  //   with clusters of top_cl CTAs; levels > top_L per level
+    bool s2m_w = false;              // S2M on k_s2m_w (complex64, M_L = 64, P % 16 == 0)
     int fs_lc1 = 0, fs_lc2 = 0, fs_lr = 0;   // four-step large-M FFT: column pass bits (2nd: 0 = none), row pass bits
     bool inverse = false;            // FMMFFT_FLAG_INVERSE: x = F_N^{-1} y
     bool real = false;               // FMMFFT_FLAG_REAL: N (below) is the complex length H = N_real / 2
@@ -901,7 +902,7 @@ struct Exec {
         const int PCs = std::min(p->P, sizeof(R) == 4 ? 32 : 16);
         constexpr int PCW = s2mw_pc<R>();
         // complex64 (complex128's S2M is DFMA-bound with Q = 24: k_s2m measured faster, 1.68 vs 2.12 ms)
-        if (sizeof(R) == 4 && p->M_L == 64 && p->P % PCW == 0 && !getenv("FMMFFT_S2M_OLD")) {   // warp-per-box S2M (k_s2m_w)
+        if (p->s2m_w) {                                  // warp-per-box S2M (k_s2m_w)
             const int Qp = (p->Q + 3) / 4 * 4;
             const long long tasks = (long long)p->nb * (p->P / PCW);
             const int bpw = (int)std::max<long long>(1, std::min<long long>(8, tasks / (S2MW_WARPS * 148 * 4)));
@@ -2096,6 +2097,8 @@ static fmmfft_status_t plan_complex(fmmfft_plan_t* plan, long long N, int P, int
     // the cluster far field gathers M^L and scatters L^L one FMM (one p) at a time: keep both
     // p-major so those are contiguous runs (debug plans keep [b][q][p] for the stage buffers)
     p->pmaj = p->tree_p && p->tree_cl > 1 && L > B && !(flags & FMMFFT_FLAG_DEBUG);
+    // complex64 only: complex128's S2M is DFMA-bound at Q = 24 (k_s2m measured faster, 1.68 vs 2.12 ms)
+    p->s2m_w = precision == FMMFFT_C64 && M_L == 64 && P % 16 == 0 && !getenv("FMMFFT_S2M_OLD");
     const char* g_env = getenv("FMMFFT_NO_GRAPH");
     p->use_graph = !(g_env && g_env[0] == '1');
     plan_mfft(p);
@@ -2269,9 +2272,11 @@ fmmfft_status_t fmmfft_get_info(fmmfft_plan_t p, fmmfft_info_t* info) {
     info->n_stages = ST_COUNT + 1; info->workspace_bytes = p->ws_bytes; info->kernels_per_execute = p->kernels;
     info->variant = (p->tree_p ? FMMFFT_VARIANT_TREE_FUSED : 0u) | (p->s2t_tc ? FMMFFT_VARIANT_S2T_TC : 0u) |
                     (p->s2t_fft ? FMMFFT_VARIANT_S2T_FFT : 0u) |
+                    (p->s2m_w ? FMMFFT_VARIANT_S2M_WARP : 0u) | (p->top_L ? FMMFFT_VARIANT_TOP_CLUSTER : 0u) |
                     (p->row_fft1 ? FMMFFT_VARIANT_ROW_FFT1 : 0u) | (p->fs_lr ? FMMFFT_VARIANT_FOURSTEP : 0u) |
                     (!p->tree_p && !p->direct ? FMMFFT_VARIANT_DOWN_LVL : 0u) |
                     (p->pmaj ? FMMFFT_VARIANT_PMAJ : 0u);
+    info->top_level = p->top_L;
     return FMMFFT_SUCCESS;
 }
 

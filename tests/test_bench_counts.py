@@ -62,3 +62,7 @@ def test_stage_flops_match_oracle_contractions(monkeypatch, N, P, B, Q, M_L):
     assert r["down"][1] == m2l_levels + fl["L2L"]
     fused = bench.stage_rooflines(N, P, B, Q, M_L, 1, L, "c64", True, False, "k")
     assert fused["top"][1] == fl["M2M"] + fl["M2L"] + fl["L2L"]
+    # wide tree with the cluster top (levels B..top_L in k_tree_pc): the three stages partition the work
+    for top_L in range(B + 1, L + 1):
+        h = bench.stage_rooflines(N, P, B, Q, M_L, 1, L, "c64", False, False, "k", top_L=top_L)
+        assert h["m2m"][1] + h["top"][1] + h["down"][1] == pytest.approx(fl["M2M"] + fl["M2L"] + fl["L2L"])
