@@ -1128,11 +1128,14 @@ struct Exec {
             const int tabB = ((1 << p->B) - 3) * p->Q * p->Q;
             // complex64, Q = 16 or 8: each FMM on a cluster of 2 CTAs (k_tree_pc)
             if constexpr (sizeof(R) == 4) {
-                if (p->tree_cl == 2) {
-                    const size_t smem = tree_pc_smem(p, 2);
-                    const unsigned grid = (unsigned)((p->P - 1) * 2);
-                    if (p->Q == 16) launch_cluster(k_tree_pc<16, 512, 2>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
-                    else            launch_cluster(k_tree_pc<8, 512, 2>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
+                if (p->tree_cl > 1) {
+                    const size_t smem = tree_pc_smem(p, p->tree_cl);
+                    const unsigned grid = (unsigned)((p->P - 1) * p->tree_cl);
+                    dispatch<2, 4, 8>(p->tree_cl, [&](auto cl) {
+                        constexpr int CL = decltype(cl)::value;
+                        if (p->Q == 16) launch_cluster(k_tree_pc<16, 512, CL>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
+                        else            launch_cluster(k_tree_pc<8, 512, CL>, grid, 512, smem, s, a, (const float*)p->m2m, p->P, tabB);
+                    });
                     LAUNCH_CHECK();
                     continue;
                 }
@@ -2062,6 +2065,7 @@ static fmmfft_status_t plan_complex(fmmfft_plan_t* plan, long long N, int P, int
         // complex64, Q = 8 / 16: each FMM's tree on a cluster of 2 CTAs (k_tree_pc); else one CTA
         // per FMM (k_tree_p)
         if (p->tree_p && precision == FMMFFT_C64 && (Q == 16 || Q == 8) && tree_pc_smem(p, 2) <= (size_t)optin) p->tree_cl = 2;
+        // (clusters of 4 measured slower at cfg2: the fused far field 29 -> 41 us)
         // wide trees at G = 1 (complex64, Q = 8 / 16): the levels below the first wide level (the
         // per-level kernels' launch-latency-bound top: k_up, k_base, k_tree_down) as ONE k_tree_pc
         // launch, each FMM's top subtree on a cluster of 8 (else 4, 2) CTAs, levels B..top_L
