@@ -915,7 +915,7 @@ k_c2r_pre_dist(const C2<R>* __restrict__ X, const C2<R>* __restrict__ Xm, const 
 // W[k2][b M_L + m] for every k2 (coalesced over m). CTA = NBX consecutive boxes x M_L threads.
 // ---------------------------------------------------------------------------------------------
 #ifndef FMMFFT_PPR_MINB
-#define FMMFFT_PPR_MINB 3            // k_post_pfft_r CTAs per SM the register budget is sized for
+#define FMMFFT_PPR_MINB 4            // k_post_pfft_r CTAs per SM the register budget is sized for (3: 252 -> 4: 240 us at cfg3)
 #endif
 template <typename R, int LP, int QT>
 __global__ void __launch_bounds__(256, FMMFFT_PPR_MINB)
