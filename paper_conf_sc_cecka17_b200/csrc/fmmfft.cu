@@ -1444,17 +1444,14 @@ struct Exec {
         if (p->P <= 32 && p->P >= 2 && (p->Q == 8 || p->Q == 16 || p->Q == 24) && p->M_L <= 256) {
             const int nbx = std::max(1, std::min(p->nb, 256 / p->M_L));
             if (p->nb % nbx == 0) {
-                const size_t smem = ((size_t)2 * nbx * p->Q * p->P + 2 * p->P + 16) * sizeof(C) + (size_t)p->Q * p->M_L * sizeof(R);
-                // groups of nbx boxes per CTA: ~2 waves of FMMFFT_PPR_MINB CTAs per SM
-                const int ngroups = p->nb / nbx;
-                const int gpc = std::max(1, ngroups / (148 * FMMFFT_PPR_MINB * 2));
+                const size_t smem = ((size_t)nbx * p->Q * p->P + 2 * p->P + 16) * sizeof(C) + (size_t)p->Q * p->M_L * sizeof(R);
                 for (RankBufs& rb : p->ranks) {
                     bool ok = dispatch<1, 2, 3, 4, 5>(ilog2(p->P), [&](auto lp) {
                         constexpr int LP = decltype(lp)::value;
                         dispatch<8, 16, 24>(p->Q, [&](auto qv) {
-                            launch_pdl(k_post_pfft_r<R, LP, decltype(qv)::value>, (unsigned)((ngroups + gpc - 1) / gpc), nbx * p->M_L,
-                                       smem, s, (const C*)rb.Tn, (const C*)rb.Lloc[p->L], (const C*)rb.r, (const C*)p->rho,
-                                       (const R*)p->s2m, (C*)rb.W, ilog2(p->M_L), (int)p->Mg, (int)p->pmaj, ngroups, gpc);
+                            launch_pdl(k_post_pfft_r<R, LP, decltype(qv)::value>, (unsigned)(p->nb / nbx), nbx * p->M_L, smem, s,
+                                       (const C*)rb.Tn, (const C*)rb.Lloc[p->L], (const C*)rb.r, (const C*)p->rho,
+                                       (const R*)p->s2m, (C*)rb.W, ilog2(p->M_L), (int)p->Mg, (int)p->pmaj);
                         });
                     });
                     if (!ok) return fail(FMMFFT_UNSUPPORTED, "k_post_pfft_r: P=%d", p->P);

@@ -912,116 +912,88 @@ k_c2r_pre_dist(const C2<R>* __restrict__ X, const C2<R>* __restrict__ Xm, const 
 // the FFT): thread (box b, m) loads T_near[p][b][.][m] for all p (coalesced over m), adds
 // L2T_{mq} L^L_{pqb} (L^L of its box broadcast from shared memory, two p per 16-byte load),
 // applies POST, runs the P-point DFT in registers (radix 2/4/8/16, 32 = 2 x 16) and stores
-// W[k2][b M_L + m] for every k2 (coalesced over m). CTA = a run of groups of NBX consecutive boxes
-// x M_L threads: the next group's T_near column (registers) and L^L (cp.async, double-buffered
-// shared memory) are in flight while the current group is computed.
+// W[k2][b M_L + m] for every k2 (coalesced over m). CTA = NBX consecutive boxes x M_L threads.
 // ---------------------------------------------------------------------------------------------
 #ifndef FMMFFT_PPR_MINB
-#define FMMFFT_PPR_MINB 2            // k_post_pfft_r CTAs per SM (128 registers: the current and the next group's column)
+#define FMMFFT_PPR_MINB 4            // k_post_pfft_r CTAs per SM the register budget is sized for (3: 252 -> 4: 240 us at cfg3)
 #endif
 template <typename R, int LP, int QT>
 __global__ void __launch_bounds__(256, FMMFFT_PPR_MINB)
 k_post_pfft_r(const C2<R>* __restrict__ Tn, const C2<R>* __restrict__ LL, const C2<R>* __restrict__ r,
-              const C2<R>* __restrict__ rho, const R* __restrict__ s2m, C2<R>* __restrict__ W, int lML, int Mg, int pmaj,
-              int ngroups, int groups_per_cta) {
+              const C2<R>* __restrict__ rho, const R* __restrict__ s2m, C2<R>* __restrict__ W, int lML, int Mg, int pmaj) {
     pdl_trigger();
     using C = C2<R>;
     constexpr int P = 1 << LP, Q = QT;
     const int M_L = 1 << lML;
     const int nbx = blockDim.x >> lML;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    C* Lsm0 = reinterpret_cast<C*>(smem_raw);                     // [2][nbx][Q][P] (double-buffered)
-    C* rr = Lsm0 + 2 * nbx * Q * P;                                // [P] r_p
+    C* Lsm = reinterpret_cast<C*>(smem_raw);                      // [nbx][Q][P]
+    C* rr = Lsm + nbx * Q * P;                                     // [P] r_p
     C* rh = rr + P;                                                // [P] rho_p
     C* tw32 = rh + P;                                              // [16] w_32^k
     R* wsm = reinterpret_cast<R*>(tw32 + 16);                      // [Q][M_L] L2T_{mq} = S2M_{qm}
     const int tid = threadIdx.x, bx = tid >> lML, m = tid & (M_L - 1);
-    const int g_begin = blockIdx.x * groups_per_cta;
-    const int g_end = min(ngroups, g_begin + groups_per_cta);
+    const int b = blockIdx.x * nbx + bx;
     for (int idx = tid; idx < Q * M_L; idx += blockDim.x) cp_async_elem(wsm + idx, s2m + idx);
     if (tid < 16) tw32[tid] = twiddle_pow2(R(0), tid, 5);
     pdl_wait();                                                   // T_near / L^L / r from the FMM stages
-    if (tid < P) { rr[tid] = ldg_c(r + tid); rh[tid] = ldg_c(rho + tid); }
-    // box group g = boxes g nbx .. g nbx + nbx - 1: L^L into Lsm0[buf] (cp.async group), T_near
-    // column of (box, m) into registers
-    auto stage_L = [&](int g, C* Lsm) {
+    {
         constexpr int V = 16 / sizeof(C);
         if (pmaj) {                                               // [p][b][q] -> Lsm[bx][p][q]
             const int nbt = Mg >> lML;
             for (int idx = tid; idx < nbx * P * Q / V; idx += blockDim.x) {
                 const int e = idx * V, row = e / Q, q = e - row * Q;  // row = bx P + p
                 const int bxx = row / P, pp = row - bxx * P;
-                cp_async<16>(Lsm + e, LL + ((size_t)pp * nbt + (size_t)g * nbx + bxx) * Q + q);
+                cp_async<16>(Lsm + e, LL + ((size_t)pp * nbt + (size_t)blockIdx.x * nbx + bxx) * Q + q);
             }
         } else {
-            const C* src = LL + (size_t)g * nbx * Q * P;
+            const C* src = LL + (size_t)blockIdx.x * nbx * Q * P;
             for (int idx = tid; idx < nbx * Q * P / V; idx += blockDim.x) cp_async<16>(Lsm + idx * V, src + idx * V);
         }
-        cp_async_commit();
-    };
-    auto load_T = [&](int g, C (&v)[P]) {
-        const R* tn = reinterpret_cast<const R*>(Tn) + ((size_t)(g * nbx + bx) << (lML + 1)) + m;
-#pragma unroll
-        for (int p = 0; p < P; ++p) {
-            v[p].x = __ldg(tn + (size_t)p * 2 * Mg);
-            v[p].y = __ldg(tn + (size_t)p * 2 * Mg + M_L);
-        }
-    };
-    C v[P], vn[P];
-    if (g_begin < g_end) {
-        stage_L(g_begin, Lsm0);
-        load_T(g_begin, v);
+        if (tid < P) { rr[tid] = ldg_c(r + tid); rh[tid] = ldg_c(rho + tid); }
     }
-    for (int g = g_begin; g < g_end; ++g) {
-        C* Lsm = Lsm0 + ((g - g_begin) & 1) * nbx * Q * P;
-        const bool more = g + 1 < g_end;
-        if (more) {                                               // next group's loads in flight meanwhile
-            stage_L(g + 1, Lsm0 + ((g + 1 - g_begin) & 1) * nbx * Q * P);
-            load_T(g + 1, vn);
-            cp_async_wait_group<1>();
-        } else {
-            cp_async_wait_group<0>();
-        }
-        __syncthreads();
-        // L2T accumulated straight into the column (q outer: one L2T coefficient register, the L^L
-        // row of q a broadcast), then POST; p = 0 is the identity (C_0 = I, R1)
-        const C* Lb = Lsm + bx * Q * P;
+    C v[P];
+    const R* tn = reinterpret_cast<const R*>(Tn) + ((size_t)b << (lML + 1)) + m;
+#pragma unroll
+    for (int p = 0; p < P; ++p) {
+        v[p].x = __ldg(tn + (size_t)p * 2 * Mg);
+        v[p].y = __ldg(tn + (size_t)p * 2 * Mg + M_L);
+    }
+    cp_async_wait_all();
+    __syncthreads();
+    // L2T accumulated straight into the column (q outer: one L2T coefficient register, the L^L
+    // row of q a broadcast), then POST; p = 0 is the identity (C_0 = I, R1)
+    const C* Lb = Lsm + bx * Q * P;
 #pragma unroll 4
-        for (int q = 0; q < Q; ++q) {
-            const R wq = wsm[q * M_L + m];
+    for (int q = 0; q < Q; ++q) {
+        const R wq = wsm[q * M_L + m];
 #pragma unroll
-            for (int p = 1; p < P; ++p) rfma(v[p], wq, pmaj ? Lb[p * Q + q] : Lb[q * P + p]);
-        }
+        for (int p = 1; p < P; ++p) rfma(v[p], wq, pmaj ? Lb[p * Q + q] : Lb[q * P + p]);
+    }
 #pragma unroll
-        for (int p = 1; p < P; ++p) {
-            C t = v[p];
-            t.x -= rr[p].y; t.y += rr[p].x;                        // + i r_p
-            v[p] = cmul(rh[p], t);
-        }
-        // P-point DFT over p, natural order
-        if constexpr (P <= 16) {
-            dft_small<P>(v);
-        } else {                                                  // 32 = 2 x 16: X[k] = E[k] + w^k O[k]
-            C e[16], o[16];
+    for (int p = 1; p < P; ++p) {
+        C t = v[p];
+        t.x -= rr[p].y; t.y += rr[p].x;                            // + i r_p
+        v[p] = cmul(rh[p], t);
+    }
+    // P-point DFT over p, natural order
+    if constexpr (P <= 16) {
+        dft_small<P>(v);
+    } else {                                                      // 32 = 2 x 16: X[k] = E[k] + w^k O[k]
+        C e[16], o[16];
 #pragma unroll
-            for (int t = 0; t < 16; ++t) { e[t] = v[2 * t]; o[t] = v[2 * t + 1]; }
-            dft16(e); dft16(o);
+        for (int t = 0; t < 16; ++t) { e[t] = v[2 * t]; o[t] = v[2 * t + 1]; }
+        dft16(e); dft16(o);
 #pragma unroll
-            for (int k = 0; k < 16; ++k) {
-                const C ow = cmul(o[k], tw32[k]);
-                v[k] = cadd(e[k], ow);
-                v[k + 16] = csub(e[k], ow);
-            }
-        }
-        C* dst = W + ((size_t)(g * nbx + bx) << lML) + m;
-#pragma unroll
-        for (int k2 = 0; k2 < P; ++k2) dst[(size_t)k2 * Mg] = v[k2];
-        __syncthreads();                                          // Lsm reused two groups later
-        if (more) {
-#pragma unroll
-            for (int p = 0; p < P; ++p) v[p] = vn[p];
+        for (int k = 0; k < 16; ++k) {
+            const C ow = cmul(o[k], tw32[k]);
+            v[k] = cadd(e[k], ow);
+            v[k + 16] = csub(e[k], ow);
         }
     }
+    C* dst = W + ((size_t)b << lML) + m;
+#pragma unroll
+    for (int k2 = 0; k2 < P; ++k2) dst[(size_t)k2 * Mg] = v[k2];
 }
 
 }  // namespace fmmfft
