@@ -243,6 +243,7 @@ struct fmmfft_plan_s {
     int top_L = 0;                   // > 0: wide tree (G = 1) whose levels B..top_L run on k_tree_pc
     int top_cl = 0;                  //   with clusters of top_cl CTAs; levels > top_L per level
     bool s2m_w = false;              // S2M on k_s2m_w (complex64, M_L = 64, P % 16 == 0)
+    bool s2m_m2m = false;            //   with the first M2M level (L -> L-1) fused into it
     int fs_lc1 = 0, fs_lc2 = 0, fs_lr = 0;   // four-step large-M FFT: column pass bits (2nd: 0 = none), row pass bits
     bool inverse = false;            // FMMFFT_FLAG_INVERSE: x = F_N^{-1} y
     bool real = false;               // FMMFFT_FLAG_REAL: N (below) is the complex length H = N_real / 2
@@ -905,12 +906,14 @@ struct Exec {
         if (p->s2m_w) {                                  // warp-per-box S2M (k_s2m_w)
             const int Qp = (p->Q + 3) / 4 * 4;
             const long long tasks = (long long)p->nb * (p->P / PCW);
-            const int bpw = (int)std::max<long long>(1, std::min<long long>(8, tasks / (S2MW_WARPS * 148 * 4)));
+            int bpw = (int)std::max<long long>(1, std::min<long long>(8, tasks / (S2MW_WARPS * 148 * 4)));
+            if (p->s2m_m2m) bpw = std::max(2, bpw & ~1);                // sibling pairs within one warp
             const dim3 grid((unsigned)((p->nb + (long long)S2MW_WARPS * bpw - 1) / ((long long)S2MW_WARPS * bpw)), (unsigned)(p->P / PCW));
             for (RankBufs& rb : p->ranks) {
                 const C* S = in[p->virt ? rb.g : 0];
                 launch_pdl(k_s2m_w<R>, grid, S2MW_WARPS * 32, s2mw_smem<R>(Qp), s, S, interior(rb.Mpad[p->L]), (const R*)p->s2mT,
-                           p->P, p->Q, (C*)rb.Sp, (C*)rb.Tn, p->nb, (int)p->pmaj, bpw);
+                           p->P, p->Q, (C*)rb.Sp, (C*)rb.Tn, p->nb, (int)p->pmaj, bpw,
+                           p->s2m_m2m ? interior(rb.Mpad[p->L - 1]) : (C*)nullptr, (const R*)p->m2m);
                 LAUNCH_CHECK();
             }
         } else
@@ -1189,7 +1192,9 @@ struct Exec {
         fmmfft_status_t st;
         for (RankBufs& rb : p->ranks) {
             auto outs = [&](int l) -> void* { return interior(rb.Mpad[l]); };
-            if ((st = launch_up(interior(rb.Mpad[p->L]), p->L, p->top_L ? p->top_L : p->lg, nb_at(p->L), outs))) return st;
+            // (the first level L -> L-1 already came out of k_s2m_w when p->s2m_m2m)
+            const int from = p->s2m_m2m ? p->L - 1 : p->L;
+            if ((st = launch_up(interior(rb.Mpad[from]), from, p->top_L ? p->top_L : p->lg, nb_at(from), outs))) return st;
         }
         return FMMFFT_SUCCESS;
     }
@@ -2103,6 +2108,10 @@ static fmmfft_status_t plan_complex(fmmfft_plan_t* plan, long long N, int P, int
     p->pmaj = p->tree_p && p->tree_cl > 1 && L > B && !(flags & FMMFFT_FLAG_DEBUG);
     // complex64 only: complex128's S2M is DFMA-bound at Q = 24 (k_s2m measured faster, 1.68 vs 2.12 ms)
     p->s2m_w = precision == FMMFFT_C64 && M_L == 64 && P % 16 == 0 && !getenv("FMMFFT_S2M_OLD");
+    // NEXT-4 kernel fusion: the first upward level from the S2M kernel's registers
+    // (saves one read of M^L and a launch); per-level trees only, levels L-1 >= the gathered / top level
+    p->s2m_m2m = p->s2m_w && !p->tree_p && !p->pmaj && L - 1 >= std::max(p->lg, p->top_L) && L - 1 >= B &&
+                 (p->nb % 2) == 0 && !getenv("FMMFFT_S2M_NOFUSE");
     const char* g_env = getenv("FMMFFT_NO_GRAPH");
     p->use_graph = !(g_env && g_env[0] == '1');
     plan_mfft(p);
