@@ -130,7 +130,7 @@ def load_traffic(workload: str, G: int, kernel: str):
 
 
 def stage_rooflines(N, P, B, Q, M_L, G, L, prec, tree_fused, s2t_tc, mfft_kernel, top_L=0, s2t_fft=False,
-                    s2m_w=False):
+                    s2m_w=False, s2m_m2m=False):
     """Algorithmic work per execute of each stage, per rank, restated from PAPER.md §5.1
     (P:1159-1174): W = flops (a complex-data x real-operator multiply-add is 2C = 4 real flops),
     D = algorithmic HBM bytes (each operand read once, each result written once). Returns
@@ -171,6 +171,15 @@ def stage_rooflines(N, P, B, Q, M_L, G, L, prec, tree_fused, s2t_tc, mfft_kernel
         out["m2m"] = ("k_m2m_lvl + k_up", m2m, 3 * up * exp_b)
         out["top"] = ("k_base", base, 2 * 2 ** B * exp_b)
         out["down"] = ("k_m2l_lvl + k_tree_down", down, 3 * dn * exp_b)
+    if s2m_m2m and "m2m" in out:
+        # the first upward level (parents at L-1) is computed inside k_s2m_w: its flops and its
+        # parent write move from the M2M stage to the S2M stage (the M^L re-read disappears)
+        par = 2 ** (L - 1) / G
+        f1 = 2 * C * fmm * Q * Q * 2 * par
+        k, W, D = out["m2m"]
+        out["m2m"] = (k, W - f1, D - 3 * par * exp_b)
+        k, W, D = out["s2m"]
+        out["s2m"] = (k, W + f1, D + par * exp_b)
     return out
 
 
@@ -293,7 +302,7 @@ def roofline_table(stages, N, P, B, Q, M_L, G, info, prec, workload, virt):
     rl = {}
     for name, (kname, W, D) in stage_rooflines(N, P, B, Q, M_L, G, info["L"], prec, bool(v & 1), s2t_tc, mk,
                                                info.get("top_level", 0) if v & 512 else 0, bool(v & 128),
-                                               bool(v & 256)).items():
+                                               bool(v & 256), bool(v & 1024)).items():
         t = stages.get(name)
         if not t or t != t:
             continue

@@ -196,6 +196,7 @@ typedef struct {
 #define FMMFFT_VARIANT_TREE_FUSED 1u  /* far field as one per-FMM kernel (G = 1, tree fits smem) */
 #define FMMFFT_VARIANT_S2T_TC     2u  /* near field on tcgen05 tensor cores (3xTF32)             */
 #define FMMFFT_VARIANT_S2M_WARP 256u  /* S2M (+ the S' copy) one warp per box (k_s2m_w)            */
+#define FMMFFT_VARIANT_S2M_M2M 1024u  /* the first M2M level (L -> L-1) fused into k_s2m_w         */
 #define FMMFFT_VARIANT_TOP_CLUSTER 512u /* wide tree (G = 1): the top levels of each FMM on a CTA
                                          cluster (k_tree_pc), the wide levels per level            */
 #define FMMFFT_VARIANT_S2T_FFT  128u  /* near field as a fast convolution: per-box DFT_128, 3

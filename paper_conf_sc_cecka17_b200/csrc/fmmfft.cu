@@ -2286,6 +2286,7 @@ fmmfft_status_t fmmfft_get_info(fmmfft_plan_t p, fmmfft_info_t* info) {
     info->variant = (p->tree_p ? FMMFFT_VARIANT_TREE_FUSED : 0u) | (p->s2t_tc ? FMMFFT_VARIANT_S2T_TC : 0u) |
                     (p->s2t_fft ? FMMFFT_VARIANT_S2T_FFT : 0u) |
                     (p->s2m_w ? FMMFFT_VARIANT_S2M_WARP : 0u) | (p->top_L ? FMMFFT_VARIANT_TOP_CLUSTER : 0u) |
+                    (p->s2m_m2m ? FMMFFT_VARIANT_S2M_M2M : 0u) |
                     (p->row_fft1 ? FMMFFT_VARIANT_ROW_FFT1 : 0u) | (p->fs_lr ? FMMFFT_VARIANT_FOURSTEP : 0u) |
                     (!p->tree_p && !p->direct ? FMMFFT_VARIANT_DOWN_LVL : 0u) |
                     (p->pmaj ? FMMFFT_VARIANT_PMAJ : 0u);

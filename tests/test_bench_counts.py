@@ -66,3 +66,6 @@ def test_stage_flops_match_oracle_contractions(monkeypatch, N, P, B, Q, M_L):
     for top_L in range(B + 1, L + 1):
         h = bench.stage_rooflines(N, P, B, Q, M_L, 1, L, "c64", False, False, "k", top_L=top_L)
         assert h["m2m"][1] + h["top"][1] + h["down"][1] == pytest.approx(fl["M2M"] + fl["M2L"] + fl["L2L"])
+        f = bench.stage_rooflines(N, P, B, Q, M_L, 1, L, "c64", False, False, "k", top_L=top_L, s2m_m2m=True)
+        assert f["s2m"][1] + f["m2m"][1] + f["top"][1] + f["down"][1] == pytest.approx(
+            fl["S2M"] + fl["M2M"] + fl["M2L"] + fl["L2L"])
