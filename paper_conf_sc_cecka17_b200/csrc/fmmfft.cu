@@ -964,6 +964,8 @@ struct Exec {
                 // over (P - 1) floor(148 / (P - 1)) CTAs, so a CTA's run stays within one p (B_p
                 // loaded once) and the few SMs left over run the far field meanwhile (measured:
                 // all 148 SMs on S2T, with B_p reloads, was 334 -> 354 us at cfg3)
+                // (fewer CTAs, leaving SMs to the far field, measured slower at cfg3: 105 CTAs 1.66 ms,
+                // 60 CTAs 1.73 ms, vs 1.64 ms)
                 const int ctas = (int)std::min<long long>((long long)(p->P - 1) * std::max(1, 148 / (p->P - 1)), work);
                 for (RankBufs& rb : p->ranks) {
                     // several tiles per CTA: A chunks prefetched two ahead; one tile: one ahead (the
