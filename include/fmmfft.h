@@ -197,6 +197,7 @@ typedef struct {
 #define FMMFFT_VARIANT_S2T_TC     2u  /* near field on tcgen05 tensor cores (3xTF32)             */
 #define FMMFFT_VARIANT_S2M_WARP 256u  /* S2M (+ the S' copy) one warp per box (k_s2m_w)            */
 #define FMMFFT_VARIANT_S2M_M2M 1024u  /* the first M2M level (L -> L-1) fused into k_s2m_w         */
+#define FMMFFT_VARIANT_S2M_SYM 2048u  /* S2M by the reflection symmetry (even / odd halves)        */
 #define FMMFFT_VARIANT_TOP_CLUSTER 512u /* wide tree (G = 1): the top levels of each FMM on a CTA
                                          cluster (k_tree_pc), the wide levels per level            */
 #define FMMFFT_VARIANT_S2T_FFT  128u  /* near field as a fast convolution: per-box DFT_128, 3

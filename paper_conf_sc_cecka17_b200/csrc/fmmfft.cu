@@ -244,6 +244,7 @@ struct fmmfft_plan_s {
     int top_cl = 0;                  //   with clusters of top_cl CTAs; levels > top_L per level
     bool s2m_w = false;              // S2M on k_s2m_w (complex64, M_L = 64, P % 16 == 0)
     bool s2m_m2m = false;            //   with the first M2M level (L -> L-1) fused into it
+    bool s2m_sym = false;            //   and the reflection-symmetric (even / odd) S2M (Q % 8 == 0)
     int fs_lc1 = 0, fs_lc2 = 0, fs_lr = 0;   // four-step large-M FFT: column pass bits (2nd: 0 = none), row pass bits
     bool inverse = false;            // FMMFFT_FLAG_INVERSE: x = F_N^{-1} y
     bool real = false;               // FMMFFT_FLAG_REAL: N (below) is the complex length H = N_real / 2
@@ -913,7 +914,7 @@ struct Exec {
                 const C* S = in[p->virt ? rb.g : 0];
                 launch_pdl(k_s2m_w<R>, grid, S2MW_WARPS * 32, s2mw_smem<R>(Qp), s, S, interior(rb.Mpad[p->L]), (const R*)p->s2mT,
                            p->P, p->Q, (C*)rb.Sp, (C*)rb.Tn, p->nb, (int)p->pmaj, bpw,
-                           p->s2m_m2m ? interior(rb.Mpad[p->L - 1]) : (C*)nullptr, (const R*)p->m2m);
+                           p->s2m_m2m ? interior(rb.Mpad[p->L - 1]) : (C*)nullptr, (const R*)p->m2m, (int)p->s2m_sym);
                 LAUNCH_CHECK();
             }
         } else
@@ -2108,7 +2109,9 @@ static fmmfft_status_t plan_complex(fmmfft_plan_t* plan, long long N, int P, int
     // the cluster far field gathers M^L and scatters L^L one FMM (one p) at a time: keep both
     // p-major so those are contiguous runs (debug plans keep [b][q][p] for the stage buffers)
     p->pmaj = p->tree_p && p->tree_cl > 1 && L > B && !(flags & FMMFFT_FLAG_DEBUG);
-    // complex64 only: complex128's S2M is DFMA-bound at Q = 24 (k_s2m measured faster, 1.68 vs 2.12 ms)
+    // complex64 only: complex128's S2M is DFMA-bound at Q = 24 (k_s2m_w measured 2.12 ms vs 1.68 ms
+    // for k_s2m; with the symmetric S2M and the fused M2M level 4.2 ms, step 21.2 -> 22.7 ms)
+    p->s2m_sym = Q % 8 == 0 && !getenv("FMMFFT_S2M_NOSYM");
     p->s2m_w = precision == FMMFFT_C64 && M_L == 64 && P % 16 == 0 && !getenv("FMMFFT_S2M_OLD");
     // NEXT-4 kernel fusion: the first upward level from the S2M kernel's registers
     // (saves one read of M^L and a launch); per-level trees only, levels L-1 >= the gathered / top level
@@ -2288,7 +2291,7 @@ fmmfft_status_t fmmfft_get_info(fmmfft_plan_t p, fmmfft_info_t* info) {
     info->variant = (p->tree_p ? FMMFFT_VARIANT_TREE_FUSED : 0u) | (p->s2t_tc ? FMMFFT_VARIANT_S2T_TC : 0u) |
                     (p->s2t_fft ? FMMFFT_VARIANT_S2T_FFT : 0u) |
                     (p->s2m_w ? FMMFFT_VARIANT_S2M_WARP : 0u) | (p->top_L ? FMMFFT_VARIANT_TOP_CLUSTER : 0u) |
-                    (p->s2m_m2m ? FMMFFT_VARIANT_S2M_M2M : 0u) |
+                    (p->s2m_m2m ? FMMFFT_VARIANT_S2M_M2M : 0u) | (p->s2m_w && p->s2m_sym ? FMMFFT_VARIANT_S2M_SYM : 0u) |
                     (p->row_fft1 ? FMMFFT_VARIANT_ROW_FFT1 : 0u) | (p->fs_lr ? FMMFFT_VARIANT_FOURSTEP : 0u) |
                     (!p->tree_p && !p->direct ? FMMFFT_VARIANT_DOWN_LVL : 0u) |
                     (p->pmaj ? FMMFFT_VARIANT_PMAJ : 0u);

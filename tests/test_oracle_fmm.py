@@ -241,3 +241,27 @@ def test_fmmfft_p_equals_2_and_structured_inputs():
     e = np.zeros(N, dtype=complex)
     e[77] = N
     assert np.max(np.abs(y - e)) < 1e-10 * N
+
+
+@pytest.mark.parametrize("Q,M_L", [(8, 64), (16, 64), (24, 64), (16, 16)])
+def test_reflection_symmetries_the_kernels_use(Q, M_L):
+    # NEXT-4: the Chebyshev nodes and the leaf points are symmetric (z -> -z,
+    # s_m -> -s_m), so S2M_{Q-1-q, m} = S2M_{q, M_L-1-m} (k_s2m_w's even / odd S2M) and
+    # M2M^+ = J M2M^- J (J = reversal); the p-shift of M2L breaks its reflection (cot(-a + t)
+    # != -cot(a + t) for t = pi p / N != 0), so M2L has none to use
+    W = O.op_S2M(Q, M_L)
+    assert np.allclose(W[::-1, ::-1], W, atol=1e-13)
+    x = np.random.default_rng(3).standard_normal(M_L) + 1j * np.random.default_rng(4).standard_normal(M_L)
+    h = M_L // 2
+    xp, xm = x[:h] + x[::-1][:h], x[:h] - x[::-1][:h]
+    Wp, Wm = (W[:, :h] + W[:, ::-1][:, :h]) / 2, (W[:, :h] - W[:, ::-1][:, :h]) / 2
+    Mq = W @ x
+    assert np.allclose(Mq[:Q // 2], (Wp @ xp + Wm @ xm)[:Q // 2], atol=1e-12)
+    assert np.allclose(Mq[::-1][:Q // 2], (Wp @ xp - Wm @ xm)[:Q // 2], atol=1e-12)
+    A = O.op_M2M(Q)
+    Am, Ap = A[:, :Q], A[:, Q:]
+    assert np.allclose(Ap, Am[::-1, ::-1], atol=1e-13)
+    N, P, lev, s = 1 << 12, 16, 3, 2
+    K = O.op_M2L(N, P, Q, lev, s)                        # [p, i, j] for FMM p + 1
+    Km = O.op_M2L(N, P, Q, lev, -s)
+    assert not np.allclose(Km[:, ::-1, ::-1], -K, atol=1e-6)
