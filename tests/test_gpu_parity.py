@@ -68,6 +68,8 @@ def rel(a, b):
     (1 << 20, 16, 4, 16, "c64", 64),       # wide tree (L = 10): per-level k_m2l_lvl for l >= 6
     (1 << 20, 16, 4, 24, "c128", 16),      # L = 12, Q = 24, fp64 k_m2l_lvl
     (1 << 20, 32, 3, 8, "c64", 32),        # L = 10, Q = 8
+    (1 << 22, 16, 4, 24, "c64", 64),       # k_s2m_w at Q = 24: 3 symmetric q quads, fused M2M, cluster top
+    (1 << 22, 32, 3, 8, "c64", 64),        # k_s2m_w at Q = 8 (one symmetric quad)
 ])
 def test_end_to_end_vs_dft(F, N, P, B, Q, prec, M_L):
     plan, x, y = run(F, N, P, B, Q, prec, M_L)
