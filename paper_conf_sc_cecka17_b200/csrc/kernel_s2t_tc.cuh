@@ -57,7 +57,12 @@ constexpr int S2TC_TAB_FLOATS_PER_P = 2 * S2TC_B_BYTES / 4;   // [k4 16][r8 48][
 // summed in the epilogue) and Alo x Bhi_s (N = 64, the same descriptor) accumulates into the first
 // 64 — 2 MMAs per (shift, component, K step) instead of 3, and A_hi is read once.
 constexpr int S2TC_B_K4N = (2 * S2TC_N / 8) * 128;         // bytes per k4 column (48 core matrices)
-constexpr int S2TC_THREADS = 288;
+#ifndef S2TC_BW
+#define S2TC_BW 8                                         // A-builder warps (4: 168 registers, S2T 369 us at cfg3; 8: 128 registers, 283 us)
+#endif
+constexpr int S2TC_BT = S2TC_BW * 32;                     // builder threads
+constexpr int S2TC_THREADS = (S2TC_BW + 5) * 32;          // builders, 4 epilogue warps, the MMA warp
+constexpr int S2TC_MMA_WARP = S2TC_BW + 4;
 
 struct S2tcSmem {                                         // byte offsets
     static constexpr int B = 0;
@@ -97,7 +102,7 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
     const size_t pblk = (size_t)nb * 64;                         // elements per p block of S' / T
 
     if (tid == 0) {
-        for (int k = 0; k < 12; ++k) tc::mbar_init(&bar[k], (k == 4 || k == 5 || k >= 10) ? 128u : 1u);
+        for (int k = 0; k < 12; ++k) tc::mbar_init(&bar[k], (k == 4 || k == 5) ? (unsigned)S2TC_BT : (k >= 10 ? 128u : 1u));
         tc::fence_barrier_init();
     }
     if (warp == 0) tc::tmem_alloc<512>(tmem_slot);
@@ -107,16 +112,16 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
     const uint32_t tmem = *tmem_slot;
     STAMP(1);
 
-    if (warp < 4) {
+    if (warp < S2TC_BW) {
         // ------------------------------------------------------------ A builders (128 threads)
-        // item j: row r = idx >> 2 (box b0 - 1 + r), k4 = idx & 3, idx = tid + 128 j < 4 x 130
-        constexpr int NJ = (4 * S2TC_ROWS + 127) / 128;          // 5
+        // item j: row r = idx >> 2 (box b0 - 1 + r), k4 = idx & 3, idx = tid + S2TC_BT j < 4 x 130
+        constexpr int NJ = (4 * S2TC_ROWS + S2TC_BT - 1) / S2TC_BT;   // 5 (3 with 8 builder warps)
         float4 sv[2][NJ][2];                                     // two chunks in flight (prefetch distance 2)
         auto load_chunk = [&](float4 (&svb)[NJ][2], int p, int t, int kc) {
             const float2* spp = Sp + (size_t)p * pblk;
 #pragma unroll
             for (int j = 0; j < NJ; ++j) {
-                const int idx = tid + 128 * j;
+                const int idx = tid + S2TC_BT * j;
                 if (idx < 4 * S2TC_ROWS) {
                     const int r = idx >> 2, k4 = idx & 3;
                     const int g = t * S2TC_BOXES - 1 + r;        // global box (within this rank)
@@ -151,7 +156,7 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
                 unsigned char* As = Asm + slot * S2TC_A_SLOT;
 #pragma unroll
                 for (int j = 0; j < NJ; ++j) {
-                    const int idx = tid + 128 * j;
+                    const int idx = tid + S2TC_BT * j;
                     if (idx < 4 * S2TC_ROWS) {
                         const int r = idx >> 2, k4 = idx & 3;
                         const float4 u0 = sv[kc & 1][j][0], u1 = sv[kc & 1][j][1];   // (re, im) of 4 consecutive m
@@ -181,7 +186,7 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
             pc = pn;
             tc_ = tn;
         }
-    } else if (warp == 8) {
+    } else if (warp == S2TC_MMA_WARP) {
         // ------------------------------------------------------------ operator loads + MMA issue
         if (lane == 0) {
             auto load_B = [&](int p) {
