@@ -49,11 +49,14 @@ def needs_build() -> bool:
     return any(os.path.getmtime(s) > t for s in sources())
 
 
+# No --split-compile: with it, nvcc's partition of the translation unit changed the register
+# allocation of unrelated kernels from build to build (k_m2l_lvl 160 vs 209 registers, k_m2m_lvl
+# 160 vs 195, measured ~3 % of the cfg3 step) — one partition gives reproducible code.
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not needs_build():
         return LIB
     cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
-           "-Xcompiler", "-fvisibility=hidden", "--expt-relaxed-constexpr", "--split-compile=8",
+           "-Xcompiler", "-fvisibility=hidden", "--expt-relaxed-constexpr",
            "-I", os.path.join(ROOT, "include"), "-I", _nccl_include(),
            os.path.join(CSRC, "fmmfft.cu"), "-o", LIB + ".tmp", "-ldl"]
     if verbose:
@@ -69,7 +72,7 @@ def build_variant(name: str, defines) -> str:
     with FMMFFT_LIB=<path>; the default library is unaffected)."""
     out = os.path.join(PKG, f"libfmmfft_{name}.so")
     cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
-           "-Xcompiler", "-fvisibility=hidden", "--expt-relaxed-constexpr", "--split-compile=8",
+           "-Xcompiler", "-fvisibility=hidden", "--expt-relaxed-constexpr",
            *[f"-D{d}" for d in defines], "-I", os.path.join(ROOT, "include"), "-I", _nccl_include(),
            os.path.join(CSRC, "fmmfft.cu"), "-o", out, "-ldl"]
     subprocess.run(cmd, check=True)
