@@ -61,14 +61,17 @@ constexpr int S2TC_B_K4N = (2 * S2TC_N / 8) * 128;         // bytes per k4 colum
 #define S2TC_BW 8                                         // A-builder warps (4: 168 registers, S2T 369 us at cfg3; 8: 128 registers, 283 us)
 #endif
 constexpr int S2TC_BT = S2TC_BW * 32;                     // builder threads
-constexpr int S2TC_THREADS = (S2TC_BW + 5) * 32;          // builders, 4 epilogue warps, the MMA warp
-constexpr int S2TC_MMA_WARP = S2TC_BW + 4;
+#ifndef S2TC_EW
+#define S2TC_EW 4                                         // epilogue warps (4, or 8: two per TMEM lane quarter)
+#endif
+constexpr int S2TC_THREADS = (S2TC_BW + S2TC_EW + 1) * 32;  // builders, epilogue warps, the MMA warp
+constexpr int S2TC_MMA_WARP = S2TC_BW + S2TC_EW;
 
 struct S2tcSmem {                                         // byte offsets
     static constexpr int B = 0;
     static constexpr int A = B + 2 * S2TC_B_BYTES;              // 2-slot ring of K chunks
     static constexpr int XT = A + 2 * S2TC_A_SLOT;              // per-warp transpose [4][32][33] floats
-    static constexpr int BAR = XT + 4 * 32 * 33 * 4;            // 12 mbarriers
+    static constexpr int BAR = XT + S2TC_EW * 32 * 33 * 4;      // 12 mbarriers
     static constexpr int TSLOT = BAR + 12 * 8;
     static constexpr int TOTAL = TSLOT + 16;
 };
@@ -102,7 +105,7 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
     const size_t pblk = (size_t)nb * 64;                         // elements per p block of S' / T
 
     if (tid == 0) {
-        for (int k = 0; k < 12; ++k) tc::mbar_init(&bar[k], (k == 4 || k == 5) ? (unsigned)S2TC_BT : (k >= 10 ? 128u : 1u));
+        for (int k = 0; k < 12; ++k) tc::mbar_init(&bar[k], (k == 4 || k == 5) ? (unsigned)S2TC_BT : (k >= 10 ? (unsigned)(S2TC_EW * 32) : 1u));
         tc::fence_barrier_init();
     }
     if (warp == 0) tc::tmem_alloc<512>(tmem_slot);
@@ -247,7 +250,8 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
         // ------------------------------------------------------------ epilogue (warps 4-7)
         // warp q reads TMEM lanes 32 q .. 32 q + 31 = boxes b0 + 32 q + lane
         const int q = warp & 3;
-        float* xt = Xt + q * 32 * 33;
+        const int eh = (warp - S2TC_BW) >> 2;                   // with 8 epilogue warps: which 2 of the 4 chunks
+        float* xt = Xt + (warp - S2TC_BW) * 32 * 33;
         for (int it = 0; it < nit; ++it) {
             const int w = w0 + it, buf = it & 1;
             const int p = w / ntile + 1, t = w - (p - 1) * ntile;
@@ -258,7 +262,7 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
             // planar [p][b][c][m]: rows of boxes b0 + 32 q + r, r < 32
             float* tw = Tn + ((size_t)p * nb + (size_t)t * S2TC_BOXES + 32 * q) * 128;
 #pragma unroll 1
-            for (int ch = 0; ch < 4; ++ch) {                     // (component, i half)
+            for (int ch = (S2TC_EW == 8 ? 2 * eh : 0); ch < (S2TC_EW == 8 ? 2 * eh + 2 : 4); ++ch) {   // (component, i half)
                 const int c = ch >> 1, h = ch & 1;
                 float v[32];
                 tc::tmem_ld32(tmem + ((uint32_t)(32 * q) << 16) + (uint32_t)(buf * 256 + c * 128 + 32 * h), v);
@@ -268,7 +272,7 @@ k_s2t_tc(const float2* __restrict__ Sp, const float2* __restrict__ haloL, const 
 #pragma unroll
                     for (int k = 0; k < 32; ++k) v[k] += v2[k];
                 }
-                if (ch == 3) {                                   // accumulators free for tile it + 2
+                if (ch == (S2TC_EW == 8 ? 2 * eh + 1 : 3)) {     // this warp's reads done: accumulators free for tile it + 2
                     tc::tc_fence_before();
                     tc::mbar_arrive(&aempty[buf]);
                 }
